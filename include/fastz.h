@@ -1,0 +1,176 @@
+/*
+ * fastz.h -- C ABI of the B200-native FastZ hot path (libfastz.so, ABI version 1).
+ *
+ * Batched gapped seed extension as in FastZ (Gundabolu, Vijaykumar, Thottethodi, SC'21; PAPER.md lines
+ * cited as P:<n>): every seed (anchor) is extended by two one-sided affine-gap Gotoh alignments,
+ * left and right of the cut point, explored under LASTZ-style y-drop pruning and
+ * traced back from the highest-scoring cell.  The work runs in the paper's two stages: a
+ * score-only inspector with eager 16x16 traceback, then a length-binned trimmed
+ * executor that writes compact traceback bits, followed by traceback walks.
+ * The exact semantics (cone reading of y-drop, tie rules, gap convention) are listed in DESIGN.md
+ * "Readings" and are bit-identical to the CPU oracle in oracle/.
+ *
+ * Conventions (all entry points):
+ *  - Return 0 (FASTZ_OK) or a negative fastz_status; fastz_strerror() describes it (thread-local detail).
+ *  - The caller owns every buffer it passes in; the library copies what it needs before returning.
+ *    The context owns its device memory (allocated through the optional dev_alloc hook or cudaMalloc).
+ *  - One context per (device, stream) user; calls on one context are not thread-safe.
+ *  - All device work is enqueued on the context's stream; fastz_extend_seeds synchronizes the stream
+ *    twice (after binning, to size the traceback pool -- P:174 "allocation at kernel launch" -- and after
+ *    the CIGAR length pass) and otherwise leaves results on the device.
+ *  - Scores are int32.  A one-sided peak score >= 2^29 sets FASTZ_FLAG_OVERFLOW on that seed.
+ */
+#ifndef FASTZ_H
+#define FASTZ_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define FASTZ_ABI_VERSION 1
+
+typedef struct fastz_ctx fastz_ctx; /* opaque */
+
+typedef enum {
+    FASTZ_OK = 0,
+    FASTZ_EINVAL = -1, /* bad argument or scoring parameter (ranges below) */
+    FASTZ_EBASE = -2,  /* a sequence character outside ACGTacgt (index in fastz_strerror text) */
+    FASTZ_ERANGE = -3, /* seed outside [0,len]; length >= 2^31; an explored band wider than the scratch */
+    FASTZ_ENOMEM = -4, /* device allocation failed */
+    FASTZ_ECUDA = -5,  /* CUDA runtime error (text in fastz_strerror) */
+    FASTZ_ETRUNC = -6, /* output buffers too small: *n_out and *cigar_bytes hold the required sizes */
+    FASTZ_ESTATE = -7  /* call out of order (e.g. get before extend) */
+} fastz_status;
+
+/*
+ * Scoring (P:70-74 recurrences; P:108 y-drop).  Defaults (fastz_default_params) are LASTZ's documented
+ * defaults -- the paper states none: HOXD70, O=400, E=30, Y=O+300E=9400, K=3000.
+ *   sub[4*a+b]  substitution score, a = target base (DP row), b = query base (column), A0 C1 G2 T3;
+ *               |sub| <= 32767.
+ *   gap_open    O in [0, 2^24]; a gap of length k costs O + k*E (s_o + s_e).
+ *   gap_extend  E in [1, 2^24].
+ *   ydrop       Y in [0, 2^28]; a cell is pruned when its score is below max(V(i-1,j), V(i,j-1)) - Y, where
+ *               V is the best score in the rectangle [0,i]x[0,j] (reading R3).
+ *   gapped_threshold  K: only sets FASTZ_FLAG_ABOVE_K; never drops a seed.
+ *   eager_max   eager-traceback window, 1..16 (16x16); sides whose peak has max(i*,j*) <= eager_max
+ *               are traced back inside the inspector and skip the executor.
+ *   dev_alloc / dev_free / alloc_user  optional device allocator hooks (e.g. a framework caching
+ *               allocator); NULL -> cudaMalloc / cudaFree.
+ */
+typedef struct {
+    int32_t sub[16];
+    int32_t gap_open;
+    int32_t gap_extend;
+    int32_t ydrop;
+    int32_t gapped_threshold;
+    int32_t eager_max;
+    int32_t reserved[3];
+    void *(*dev_alloc)(size_t bytes, void *stream, void *user);
+    void (*dev_free)(void *ptr, void *stream, void *user);
+    void *alloc_user;
+} fastz_params;
+
+/* A seed is a cut point: the right extension starts at T[tpos], Q[qpos]; the left one at T[tpos-1],
+ * Q[qpos-1] going backwards.  0 <= tpos <= tlen, 0 <= qpos <= qlen. */
+typedef struct {
+    int64_t tpos, qpos;
+} fastz_seed;
+
+#define FASTZ_FLAG_ABOVE_K 1u   /* score >= gapped_threshold */
+#define FASTZ_FLAG_LEFT_EAGER 2u  /* left side traced back eagerly in the inspector */
+#define FASTZ_FLAG_RIGHT_EAGER 4u /* right side traced back eagerly */
+#define FASTZ_FLAG_OVERFLOW 8u  /* a one-sided peak score reached 2^29 */
+
+/* One alignment per seed, in seed order (64 bytes). */
+typedef struct {
+    int32_t score;        /* left_score + right_score */
+    int32_t left_score;   /* one-sided peak scores (>= 0: the cut point itself scores 0) */
+    int32_t right_score;
+    uint32_t flags;       /* FASTZ_FLAG_* */
+    int64_t t_start, t_end; /* half-open, 0-based, forward strand: [tpos - i_L, tpos + i_R) */
+    int64_t q_start, q_end; /* [qpos - j_L, qpos + j_R) */
+    int64_t cigar_off;    /* offset of this seed's CIGAR text in the cigar buffer */
+    int32_t cigar_len;    /* bytes, no terminator; "" for an empty alignment */
+    int32_t reserved;
+} fastz_alignment;
+
+/* Fill *p with the defaults above.  Never fails. */
+void fastz_default_params(fastz_params *p);
+
+/*
+ * Create a context on `device` using `cuda_stream` (a cudaStream_t; NULL -> the library creates its own
+ * non-blocking stream).  `target`/`query` are ASCII (ACGTacgt) of tlen/qlen bytes, host or device memory
+ * (detected with cudaPointerGetAttributes); they are copied, validated and packed to 2 bits per base
+ * (forward and reversed copies) on the device.  Errors: EINVAL (NULL pointers, bad params), ERANGE (a length
+ * < 0 or >= 2^31), EBASE (invalid character), ENOMEM, ECUDA.  On error *out is NULL.
+ */
+int fastz_create(const fastz_params *p, const char *target, int64_t tlen, const char *query, int64_t qlen,
+                 int device, void *cuda_stream, fastz_ctx **out);
+
+/*
+ * Extend n seeds (host or device memory as `seeds_on_device` says; n may be 0).  Runs inspector, binning,
+ * executor, traceback and CIGAR assembly on the context's stream; results stay on the device until
+ * fastz_get_alignments.  Replaces the results of any previous call.  Errors: EINVAL, ERANGE (a seed out of
+ * range -- index in fastz_strerror -- or an explored band wider than the per-warp scratch), ENOMEM, ECUDA.
+ */
+int fastz_extend_seeds(fastz_ctx *c, const fastz_seed *seeds, int64_t n, int seeds_on_device);
+
+/*
+ * Copy the last batch's results to host memory: out[0..n) (n = seeds of the last extend call) and the
+ * concatenated CIGAR text (SAM M/I/D, target = reference).  If out_cap < n or cigar_cap < total bytes,
+ * nothing is copied, *n_out / *cigar_bytes receive the required sizes and FASTZ_ETRUNC is returned.
+ * Synchronizes the stream.  ESTATE before any extend call.
+ */
+int fastz_get_alignments(fastz_ctx *c, fastz_alignment *out, int64_t out_cap, char *cigar, int64_t cigar_cap,
+                         int64_t *n_out, int64_t *cigar_bytes);
+
+/*
+ * Device-resident view of the last batch (valid until the next extend/destroy): records and CIGAR text in
+ * the context's device memory, for callers that keep results on the GPU (e.g. a NCCL gather).
+ */
+int fastz_get_alignments_device(fastz_ctx *c, const fastz_alignment **recs, const char **cigar, int64_t *n,
+                                int64_t *cigar_bytes);
+
+/*
+ * Per-side inspector results of the last batch, side index 2*s (left) and 2*s+1 (right) for seed s:
+ * peak score, i* (target offset), j* (query offset) and side flags (bit 0 eager, bit 1 overflow).
+ * Arrays of at least 2n entries (any may be NULL).  Synchronizes.  ESTATE before extend, ETRUNC if cap < 2n.
+ */
+int fastz_get_sides(fastz_ctx *c, int32_t *score, int32_t *ti, int32_t *qj, uint32_t *flags, int64_t cap);
+
+/*
+ * Explored-cell census of the last batch: re-runs the inspector's DP in a counting variant and writes the
+ * number of explored cells of each side (the origin plus every cell with a live diagonal, upper or left
+ * neighbour -- the GCUPS numerator) into cells[2n].  Not part of the extension; synchronizes.
+ */
+int fastz_census(fastz_ctx *c, int64_t *cells, int64_t cap);
+
+/* Stage timings (ms, CUDA events on the stream) and work counts of the last extend call. */
+typedef struct {
+    float ms_total, ms_upload, ms_inspect, ms_bin, ms_execute, ms_traceback, ms_combine;
+    int32_t n_warp_slots;
+    int64_t n_seeds, n_sides, n_eager_sides, n_exec_sides;
+    int64_t bin_counts[8];        /* per side: bin 0 = eager (<=16), 1 <=512, 2 <=2048, 3 <=8192, 4 <=32768,
+                                     5 <=131072, 6 larger (4x rule) */
+    int64_t exec_words;           /* 32-bit traceback-code words written by the executor */
+    int64_t cigar_bytes;
+} fastz_stats;
+int fastz_get_stats(fastz_ctx *c, fastz_stats *s);
+
+/* Release everything; NULL-safe. */
+void fastz_destroy(fastz_ctx *c);
+
+/* Static text for a status code, plus the detail of the last error on this thread. */
+const char *fastz_strerror(int status);
+
+/* INT32 peak microbenchmark (roofline denominator): runs independent integer max/add chains on every SM
+ * for ~`ms` milliseconds on `device` and reports integer lane-operations per second. */
+int fastz_int_peak(int device, float ms, double *ops_per_s, double *sm_clock_mhz);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* FASTZ_H */

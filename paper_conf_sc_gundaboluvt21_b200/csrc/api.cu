@@ -1,0 +1,516 @@
+// api.cu -- host side of libfastz.so: the C ABI of include/fastz.h.
+//
+// Pipeline of fastz_extend_seeds (one stream, two host syncs):
+//   seeds H2D -> validate -> inspector (persistent warps, eager traceback inside) -> binning + exclusive
+//   scans of the executor sizes (static allocation from inspector sizes) -> [sync: D2H of 8 totals,
+//   grow the traceback pool] -> executor (trimmed, larger bins first) -> traceback -> CIGAR length pass +
+//   scan -> [sync: CIGAR bytes] -> CIGAR/record write.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <climits>
+#include <cstdio>
+#include <cstring>
+#include <string>
+
+#include "../../include/fastz.h"
+#include "internal.h"
+
+using namespace fz;
+
+namespace {
+
+thread_local std::string g_err;
+
+int fail(int code, const std::string& msg) {
+    g_err = msg;
+    return code;
+}
+
+#define CK(x)                                                                                  \
+    do {                                                                                       \
+        cudaError_t _e = (x);                                                                  \
+        if (_e != cudaSuccess)                                                                 \
+            return fail(_e == cudaErrorMemoryAllocation ? FASTZ_ENOMEM : FASTZ_ECUDA,          \
+                        std::string(#x) + ": " + cudaGetErrorString(_e));                       \
+    } while (0)
+
+struct DBuf {
+    void* p = nullptr;
+    size_t cap = 0;
+};
+
+}  // namespace
+
+struct fastz_ctx {
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    fastz_params prm{};
+    DevParams dp{};
+    int tlen = 0, qlen = 0;
+    DBuf Tf, Tr, Qf, Qr, stage;
+    DBuf seeds, score, ti, qj, flags, eops, bound;
+    DBuf woff, soff, roff, bin, list, counters, totals, tmpa, tmpb, tmpc, scan_tmp;
+    DBuf codes, stab, runs, nruns, ciglen, cigar, recs, cells, ring, small;
+    int R = 4, grid = 0, nslots = 0, rmask = 0;
+    int64_t n = 0, cigar_bytes = 0, nexec = 0;
+    bool have = false;
+    fastz_stats stats{};
+    cudaEvent_t ev[8] = {};
+    bool ev_ok = false;
+};
+
+namespace {
+
+int dalloc(fastz_ctx* c, DBuf& b, size_t bytes) {
+    if (bytes <= b.cap && b.p) return 0;
+    size_t want = std::max<size_t>(bytes + bytes / 4, 256);
+    if (b.p) {
+        cudaStreamSynchronize(c->stream);
+        if (c->prm.dev_free) c->prm.dev_free(b.p, c->stream, c->prm.alloc_user);
+        else cudaFree(b.p);
+        b.p = nullptr;
+        b.cap = 0;
+    }
+    void* p = nullptr;
+    if (c->prm.dev_alloc) {
+        p = c->prm.dev_alloc(want, c->stream, c->prm.alloc_user);
+        if (!p) return fail(FASTZ_ENOMEM, "dev_alloc hook returned NULL for " + std::to_string(want) + " bytes");
+    } else {
+        cudaError_t e = cudaMalloc(&p, want);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return fail(FASTZ_ENOMEM, "cudaMalloc(" + std::to_string(want) + "): " + cudaGetErrorString(e));
+        }
+    }
+    b.p = p;
+    b.cap = want;
+    return 0;
+}
+
+void dfree(fastz_ctx* c, DBuf& b) {
+    if (!b.p) return;
+    if (c->prm.dev_free) c->prm.dev_free(b.p, c->stream, c->prm.alloc_user);
+    else cudaFree(b.p);
+    b.p = nullptr;
+    b.cap = 0;
+}
+
+#define AL(buf, bytes)                               \
+    do {                                             \
+        int _r = dalloc(c, c->buf, (size_t)(bytes)); \
+        if (_r) return _r;                           \
+    } while (0)
+
+template <class T>
+T* P_(DBuf& b) {
+    return reinterpret_cast<T*>(b.p);
+}
+
+bool is_device_ptr(const void* p) {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+int check_params(const fastz_params* p) {
+    if (!p) return fail(FASTZ_EINVAL, "params is NULL");
+    for (int k = 0; k < 16; ++k)
+        if (p->sub[k] < -32767 || p->sub[k] > 32767) return fail(FASTZ_EINVAL, "|sub| must be <= 32767");
+    if (p->gap_open < 0 || p->gap_open > (1 << 24)) return fail(FASTZ_EINVAL, "gap_open must be in [0, 2^24]");
+    if (p->gap_extend < 1 || p->gap_extend > (1 << 24)) return fail(FASTZ_EINVAL, "gap_extend must be in [1, 2^24]");
+    if (p->ydrop < 0 || p->ydrop > (1 << 28)) return fail(FASTZ_EINVAL, "ydrop must be in [0, 2^28]");
+    if (p->eager_max < 1 || p->eager_max > 16) return fail(FASTZ_EINVAL, "eager_max must be in [1, 16]");
+    return 0;
+}
+
+int upload_seq(fastz_ctx* c, const char* src, int64_t len, DBuf& fwd, DBuf& rev, int64_t base_index) {
+    const size_t words = (size_t)((len + 15) / 16) + 4;
+    int r;
+    if ((r = dalloc(c, fwd, words * 4))) return r;
+    if ((r = dalloc(c, rev, words * 4))) return r;
+    CK(cudaMemsetAsync(fwd.p, 0, words * 4, c->stream));
+    CK(cudaMemsetAsync(rev.p, 0, words * 4, c->stream));
+    if (len == 0) return 0;
+    const char* dsrc = src;
+    if (!is_device_ptr(src)) {
+        if ((r = dalloc(c, c->stage, (size_t)len))) return r;
+        CK(cudaMemcpyAsync(c->stage.p, src, (size_t)len, cudaMemcpyHostToDevice, c->stream));
+        dsrc = P_<char>(c->stage);
+    }
+    if ((r = dalloc(c, c->small, 64))) return r;
+    long long init = LLONG_MAX;
+    CK(cudaMemcpyAsync(c->small.p, &init, sizeof(init), cudaMemcpyHostToDevice, c->stream));
+    CK(launch_pack(dsrc, len, P_<uint32_t>(fwd), P_<uint32_t>(rev), P_<long long>(c->small), c->stream));
+    long long bad = 0;
+    CK(cudaMemcpyAsync(&bad, c->small.p, sizeof(bad), cudaMemcpyDeviceToHost, c->stream));
+    CK(cudaStreamSynchronize(c->stream));
+    if (bad != LLONG_MAX)
+        return fail(FASTZ_EBASE, "invalid base character at index " + std::to_string(base_index + bad) +
+                                     (base_index ? " (query offset " + std::to_string(bad) + ")" : " (target)"));
+    return 0;
+}
+
+int next_pow2(int64_t v) {
+    int64_t p = 1;
+    while (p < v) p <<= 1;
+    return (int)p;
+}
+
+Batch make_batch(fastz_ctx* c) {
+    Batch b;
+    b.Tf = P_<uint32_t>(c->Tf);
+    b.Tr = P_<uint32_t>(c->Tr);
+    b.Qf = P_<uint32_t>(c->Qf);
+    b.Qr = P_<uint32_t>(c->Qr);
+    b.tlen = c->tlen;
+    b.qlen = c->qlen;
+    b.seeds = P_<long long>(c->seeds);
+    b.nseeds = (int)c->n;
+    return b;
+}
+
+SideArrays make_sides(fastz_ctx* c) {
+    SideArrays s;
+    s.score = P_<int>(c->score);
+    s.ti = P_<int>(c->ti);
+    s.qj = P_<int>(c->qj);
+    s.flags = P_<uint32_t>(c->flags);
+    s.eops = P_<unsigned long long>(c->eops);
+    s.bound = P_<long long>(c->bound);
+    return s;
+}
+
+ExecPlan make_plan(fastz_ctx* c) {
+    ExecPlan p;
+    p.woff = P_<long long>(c->woff);
+    p.soff = P_<long long>(c->soff);
+    p.roff = P_<long long>(c->roff);
+    p.bin = P_<int>(c->bin);
+    p.list = P_<int>(c->list);
+    p.counters = P_<int>(c->counters);
+    p.totals = P_<long long>(c->totals);
+    return p;
+}
+
+Outputs make_out(fastz_ctx* c) {
+    Outputs o;
+    o.codes = P_<uint32_t>(c->codes);
+    o.stab = P_<int2>(c->stab);
+    o.runs = P_<uint32_t>(c->runs);
+    o.nruns = P_<int>(c->nruns);
+    o.cig_len = P_<long long>(c->ciglen);
+    o.cigar = P_<char>(c->cigar);
+    o.recs = c->recs.p;
+    return o;
+}
+
+int ensure_ring(fastz_ctx* c) {
+    if (c->ring.p) return 0;
+    int r;
+    const size_t bytes = (size_t)c->nslots * (size_t)(c->rmask + 1) * sizeof(int4);
+    if ((r = dalloc(c, c->ring, bytes))) return r;
+    return 0;
+}
+
+}  // namespace
+
+extern "C" {
+
+void fastz_default_params(fastz_params* p) {
+    static const int32_t hoxd70[16] = {91, -114, -31, -123, -114, 100, -125, -31,
+                                       -31, -125, 100, -114, -123, -31, -114, 91};
+    memset(p, 0, sizeof(*p));
+    memcpy(p->sub, hoxd70, sizeof(hoxd70));
+    p->gap_open = 400;
+    p->gap_extend = 30;
+    p->ydrop = 9400;
+    p->gapped_threshold = 3000;
+    p->eager_max = 16;
+}
+
+const char* fastz_strerror(int status) {
+    static thread_local std::string s;
+    const char* base = "unknown status";
+    switch (status) {
+        case FASTZ_OK: base = "ok"; break;
+        case FASTZ_EINVAL: base = "invalid argument"; break;
+        case FASTZ_EBASE: base = "invalid base character"; break;
+        case FASTZ_ERANGE: base = "value out of range"; break;
+        case FASTZ_ENOMEM: base = "out of device memory"; break;
+        case FASTZ_ECUDA: base = "CUDA error"; break;
+        case FASTZ_ETRUNC: base = "output buffer too small"; break;
+        case FASTZ_ESTATE: base = "call out of order"; break;
+    }
+    s = base;
+    if (status != FASTZ_OK && !g_err.empty()) s += ": " + g_err;
+    return s.c_str();
+}
+
+void fastz_destroy(fastz_ctx* c) {
+    if (!c) return;
+    cudaSetDevice(c->device);
+    if (c->stream) cudaStreamSynchronize(c->stream);
+    DBuf* bufs[] = {&c->Tf, &c->Tr, &c->Qf, &c->Qr, &c->stage, &c->seeds, &c->score, &c->ti, &c->qj,
+                    &c->flags, &c->eops, &c->bound, &c->woff, &c->soff, &c->roff, &c->bin, &c->list,
+                    &c->counters, &c->totals, &c->tmpa, &c->tmpb, &c->tmpc, &c->scan_tmp, &c->codes,
+                    &c->stab, &c->runs, &c->nruns, &c->ciglen, &c->cigar, &c->recs, &c->cells, &c->ring,
+                    &c->small};
+    for (DBuf* b : bufs) dfree(c, *b);
+    if (c->ev_ok)
+        for (auto& e : c->ev) cudaEventDestroy(e);
+    if (c->own_stream && c->stream) cudaStreamDestroy(c->stream);
+    delete c;
+}
+
+int fastz_create(const fastz_params* p, const char* target, int64_t tlen, const char* query, int64_t qlen,
+                 int device, void* cuda_stream, fastz_ctx** out) {
+    if (!out) return fail(FASTZ_EINVAL, "out is NULL");
+    *out = nullptr;
+    int r;
+    if ((r = check_params(p))) return r;
+    if ((!target && tlen > 0) || (!query && qlen > 0)) return fail(FASTZ_EINVAL, "sequence pointer is NULL");
+    if (tlen < 0 || qlen < 0 || tlen >= (1LL << 31) || qlen >= (1LL << 31))
+        return fail(FASTZ_ERANGE, "sequence lengths must be in [0, 2^31)");
+    CK(cudaSetDevice(device));
+    fastz_ctx* c = new fastz_ctx();
+    c->device = device;
+    c->prm = *p;
+    if (cuda_stream) {
+        c->stream = (cudaStream_t)cuda_stream;
+    } else {
+        cudaError_t e = cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking);
+        if (e != cudaSuccess) {
+            delete c;
+            return fail(FASTZ_ECUDA, std::string("cudaStreamCreate: ") + cudaGetErrorString(e));
+        }
+        c->own_stream = true;
+    }
+    // column profiles (int16 pairs) per query base; profile 4 = zeros (column 0 / the origin)
+    for (int b = 0; b < 4; ++b) {
+        c->dp.cp[2 * b] = (p->sub[4 * 0 + b] & 0xffff) | (p->sub[4 * 1 + b] << 16);
+        c->dp.cp[2 * b + 1] = (p->sub[4 * 2 + b] & 0xffff) | (p->sub[4 * 3 + b] << 16);
+    }
+    c->dp.cp[8] = c->dp.cp[9] = 0;
+    c->dp.O = p->gap_open;
+    c->dp.E = p->gap_extend;
+    c->dp.Y = p->ydrop;
+    c->dp.OE = p->gap_open + p->gap_extend;
+    c->dp.K = p->gapped_threshold;
+    c->dp.eager_max = p->eager_max;
+    c->tlen = (int)tlen;
+    c->qlen = (int)qlen;
+    if ((r = upload_seq(c, target, tlen, c->Tf, c->Tr, 0)) || (r = upload_seq(c, query, qlen, c->Qf, c->Qr, tlen))) {
+        fastz_destroy(c);
+        return r;
+    }
+    dfree(c, c->stage);
+    c->R = pick_R();
+    int sms = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+    c->grid = sms * inspector_blocks_per_sm(c->R);
+    c->nslots = c->grid * WARPS;
+    // per-warp boundary ring: the widest explored band is bounded by the query side length; capped
+    int64_t want = std::max<int64_t>(std::max<int64_t>(tlen, qlen) + 64, 1024);
+    c->rmask = next_pow2(std::min<int64_t>(want, 1 << 15)) - 1;
+    for (auto& e : c->ev) cudaEventCreate(&e);
+    c->ev_ok = true;
+    *out = c;
+    return 0;
+}
+
+int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int seeds_on_device) {
+    if (!c) return fail(FASTZ_EINVAL, "ctx is NULL");
+    if (n < 0 || n > (1 << 29)) return fail(FASTZ_ERANGE, "n must be in [0, 2^29]");
+    if (n > 0 && !seeds) return fail(FASTZ_EINVAL, "seeds is NULL");
+    CK(cudaSetDevice(c->device));
+    c->have = false;
+    c->n = n;
+    const int64_t ns = 2 * n;
+    cudaStream_t st = c->stream;
+    int r;
+    if ((r = ensure_ring(c))) return r;
+    AL(seeds, std::max<int64_t>(n, 1) * 16);
+    AL(score, std::max<int64_t>(ns, 1) * 4);
+    AL(ti, std::max<int64_t>(ns, 1) * 4);
+    AL(qj, std::max<int64_t>(ns, 1) * 4);
+    AL(flags, std::max<int64_t>(ns, 1) * 4);
+    AL(eops, std::max<int64_t>(ns, 1) * 8);
+    AL(bound, std::max<int64_t>(ns, 1) * 8);
+    AL(woff, std::max<int64_t>(ns, 1) * 8);
+    AL(soff, std::max<int64_t>(ns, 1) * 8);
+    AL(roff, std::max<int64_t>(ns, 1) * 8);
+    AL(bin, std::max<int64_t>(ns, 1) * 4);
+    AL(list, std::max<int64_t>(ns, 1) * 4);
+    AL(tmpa, std::max<int64_t>(ns, 1) * 8);
+    AL(tmpb, std::max<int64_t>(ns, 1) * 8);
+    AL(tmpc, std::max<int64_t>(ns, 1) * 8);
+    AL(nruns, std::max<int64_t>(ns, 1) * 4);
+    AL(ciglen, std::max<int64_t>(2 * n, 1) * 8);
+    AL(recs, std::max<int64_t>(n, 1) * sizeof(fastz_alignment));
+    AL(counters, 64 * 4);
+    AL(totals, 8 * 8);
+    AL(small, 64);
+    const size_t stb = scan_tmp_bytes((int)std::max<int64_t>(ns, 1));
+    AL(scan_tmp, stb);
+
+    CK(cudaEventRecord(c->ev[0], st));
+    if (n > 0)
+        CK(cudaMemcpyAsync(c->seeds.p, seeds, (size_t)n * 16,
+                           seeds_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, st));
+    CK(cudaMemsetAsync(c->counters.p, 0, 64 * 4, st));
+    long long init = LLONG_MAX;
+    CK(cudaMemcpyAsync(c->small.p, &init, sizeof(init), cudaMemcpyHostToDevice, st));
+    Batch b = make_batch(c);
+    CK(launch_validate_seeds(b.seeds, b.nseeds, b.tlen, b.qlen, P_<long long>(c->small), st));
+    CK(cudaEventRecord(c->ev[1], st));
+
+    SideArrays sa = make_sides(c);
+    ExecPlan pl = make_plan(c);
+    int* counters = P_<int>(c->counters);
+    CK(launch_inspect(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, &counters[0], st));
+    CK(cudaEventRecord(c->ev[2], st));
+    CK(launch_bin(c->R, sa, (int)ns, pl, c->scan_tmp.p, stb, P_<long long>(c->tmpa), P_<long long>(c->tmpb),
+                  P_<long long>(c->tmpc), st));
+    CK(cudaEventRecord(c->ev[3], st));
+
+    // host sync 1: sizes of the executor's traceback pool
+    struct {
+        long long totals[4];
+        int counters[24];
+        long long bad;
+    } h;
+    CK(cudaMemcpyAsync(h.totals, c->totals.p, sizeof(h.totals), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(h.counters, c->counters.p, sizeof(h.counters), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(&h.bad, c->small.p, sizeof(h.bad), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (h.bad != LLONG_MAX) return fail(FASTZ_ERANGE, "seed " + std::to_string(h.bad) + " lies outside the sequences");
+    if (h.counters[20]) return fail(FASTZ_ERANGE, "an explored band is wider than the per-warp boundary ring");
+    const long long words = h.totals[0], strips = h.totals[1], nrun = h.totals[2];
+    c->nexec = h.totals[3];
+    AL(codes, std::max<long long>(words, 1) * 4);
+    AL(stab, std::max<long long>(strips, 1) * 8);
+    AL(runs, std::max<long long>(nrun, 1) * 4);
+    Outputs o = make_out(c);
+    CK(launch_execute(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, (int)c->nexec, o, st));
+    CK(cudaEventRecord(c->ev[4], st));
+    CK(launch_traceback(c->R, sa, pl, (int)c->nexec, o, st));
+    CK(cudaEventRecord(c->ev[5], st));
+    long long* dtotal = P_<long long>(c->small) + 1;
+    CK(launch_combine_len(c->dp, b, sa, pl, o, c->scan_tmp.p, stb, dtotal, st));
+    long long ctot = 0;
+    CK(cudaMemcpyAsync(&ctot, dtotal, sizeof(ctot), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));  // host sync 2: CIGAR bytes
+    AL(cigar, std::max<long long>(ctot, 1));
+    o = make_out(c);
+    CK(launch_combine_write(c->dp, b, sa, pl, o, st));
+    CK(cudaEventRecord(c->ev[6], st));
+    c->cigar_bytes = ctot;
+
+    fastz_stats& S = c->stats;
+    memset(&S, 0, sizeof(S));
+    S.n_warp_slots = c->nslots;
+    S.n_seeds = n;
+    S.n_sides = ns;
+    S.n_exec_sides = c->nexec;
+    S.n_eager_sides = h.counters[2];
+    for (int k = 0; k < 7; ++k) S.bin_counts[k] = h.counters[2 + k];
+    S.exec_words = words;
+    S.cigar_bytes = ctot;
+    c->have = true;
+    return 0;
+}
+
+int fastz_get_alignments(fastz_ctx* c, fastz_alignment* out, int64_t out_cap, char* cigar, int64_t cigar_cap,
+                         int64_t* n_out, int64_t* cigar_bytes) {
+    if (!c) return fail(FASTZ_EINVAL, "ctx is NULL");
+    if (!c->have) return fail(FASTZ_ESTATE, "no results: call fastz_extend_seeds first");
+    CK(cudaSetDevice(c->device));
+    if (n_out) *n_out = c->n;
+    if (cigar_bytes) *cigar_bytes = c->cigar_bytes;
+    if (out_cap < c->n || cigar_cap < c->cigar_bytes) return fail(FASTZ_ETRUNC, "output buffers too small");
+    if ((c->n && !out) || (c->cigar_bytes && !cigar)) return fail(FASTZ_EINVAL, "output pointer is NULL");
+    if (c->n) CK(cudaMemcpyAsync(out, c->recs.p, (size_t)c->n * sizeof(fastz_alignment), cudaMemcpyDeviceToHost, c->stream));
+    if (c->cigar_bytes) CK(cudaMemcpyAsync(cigar, c->cigar.p, (size_t)c->cigar_bytes, cudaMemcpyDeviceToHost, c->stream));
+    CK(cudaStreamSynchronize(c->stream));
+    return 0;
+}
+
+int fastz_get_alignments_device(fastz_ctx* c, const fastz_alignment** recs, const char** cigar, int64_t* n,
+                                int64_t* cigar_bytes) {
+    if (!c) return fail(FASTZ_EINVAL, "ctx is NULL");
+    if (!c->have) return fail(FASTZ_ESTATE, "no results: call fastz_extend_seeds first");
+    if (recs) *recs = reinterpret_cast<const fastz_alignment*>(c->recs.p);
+    if (cigar) *cigar = P_<char>(c->cigar);
+    if (n) *n = c->n;
+    if (cigar_bytes) *cigar_bytes = c->cigar_bytes;
+    return 0;
+}
+
+int fastz_get_sides(fastz_ctx* c, int32_t* score, int32_t* ti, int32_t* qj, uint32_t* flags, int64_t cap) {
+    if (!c) return fail(FASTZ_EINVAL, "ctx is NULL");
+    if (!c->have) return fail(FASTZ_ESTATE, "no results: call fastz_extend_seeds first");
+    if (cap < 2 * c->n) return fail(FASTZ_ETRUNC, "cap < 2n");
+    CK(cudaSetDevice(c->device));
+    const size_t bytes = (size_t)(2 * c->n) * 4;
+    if (bytes) {
+        if (score) CK(cudaMemcpyAsync(score, c->score.p, bytes, cudaMemcpyDeviceToHost, c->stream));
+        if (ti) CK(cudaMemcpyAsync(ti, c->ti.p, bytes, cudaMemcpyDeviceToHost, c->stream));
+        if (qj) CK(cudaMemcpyAsync(qj, c->qj.p, bytes, cudaMemcpyDeviceToHost, c->stream));
+        if (flags) CK(cudaMemcpyAsync(flags, c->flags.p, bytes, cudaMemcpyDeviceToHost, c->stream));
+    }
+    CK(cudaStreamSynchronize(c->stream));
+    if (flags)
+        for (int64_t k = 0; k < 2 * c->n; ++k) flags[k] &= 0xffu;
+    return 0;
+}
+
+int fastz_census(fastz_ctx* c, int64_t* cells, int64_t cap) {
+    if (!c) return fail(FASTZ_EINVAL, "ctx is NULL");
+    if (!c->have) return fail(FASTZ_ESTATE, "no results: call fastz_extend_seeds first");
+    if (cap < 2 * c->n) return fail(FASTZ_ETRUNC, "cap < 2n");
+    CK(cudaSetDevice(c->device));
+    AL(cells, std::max<int64_t>(2 * c->n, 1) * 8);
+    CK(cudaMemsetAsync(c->counters.p, 0, 4, c->stream));
+    Batch b = make_batch(c);
+    CK(launch_census(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, P_<long long>(c->cells),
+                     P_<int>(c->counters), c->stream));
+    if (c->n) CK(cudaMemcpyAsync(cells, c->cells.p, (size_t)(2 * c->n) * 8, cudaMemcpyDeviceToHost, c->stream));
+    CK(cudaStreamSynchronize(c->stream));
+    for (int64_t k = 0; k < 2 * c->n; ++k)
+        if (cells[k] < 0) return fail(FASTZ_ERANGE, "an explored band is wider than the per-warp boundary ring");
+    return 0;
+}
+
+int fastz_get_stats(fastz_ctx* c, fastz_stats* s) {
+    if (!c || !s) return fail(FASTZ_EINVAL, "NULL argument");
+    if (!c->have) return fail(FASTZ_ESTATE, "no results: call fastz_extend_seeds first");
+    CK(cudaEventSynchronize(c->ev[6]));
+    fastz_stats& S = c->stats;
+    auto el = [&](int a, int b) {
+        float ms = 0;
+        cudaEventElapsedTime(&ms, c->ev[a], c->ev[b]);
+        return ms;
+    };
+    S.ms_upload = el(0, 1);
+    S.ms_inspect = el(1, 2);
+    S.ms_bin = el(2, 3);
+    S.ms_execute = el(3, 4);
+    S.ms_traceback = el(4, 5);
+    S.ms_combine = el(5, 6);
+    S.ms_total = el(0, 6);
+    *s = S;
+    return 0;
+}
+
+int fastz_int_peak(int device, float ms, double* ops_per_s, double* sm_clock_mhz) {
+    if (!ops_per_s || !sm_clock_mhz) return fail(FASTZ_EINVAL, "NULL argument");
+    CK(int_peak_run(device, ms, ops_per_s, sm_clock_mhz));
+    return 0;
+}
+
+}  // extern "C"

@@ -1,0 +1,76 @@
+// dp.cuh -- the warp-strip y-drop DP shared by the inspector, the executor and the census (sm_100a).
+//
+// One warp computes one one-sided extension ("a single seed extension DP task to a warp").  The
+// DP matrix (rows i = target side A_1..A_M, columns j = query side B_1..B_N) is cut into horizontal
+// strips of H = 32*R rows; lane l owns R consecutive rows of the strip and holds their S/I/V state in
+// registers (the paper's cyclic use-and-discard buffers, re-designed: registers per ROW, not
+// per diagonal).  The warp sweeps the strip's columns as a skewed wavefront (lane l lags l columns, the
+// anti-diagonal layout of P:124 realised in time rather than in memory); each step every lane updates its
+// R cells of one column and hands its bottom row (X, D, W) to lane l+1 with three SHFLs ("register
+// exchange").  Only the strip's last row leaves the registers: lane 31 streams it to a per-warp ring in
+// global memory (L2-resident) and lane 0 of the next strip reads it back ("boundary cells ... written
+// out to memory to be re-loaded later for the next strip").
+//
+// Arithmetic: X = S - (O+E) is carried instead of S, so the gap opens of the cell below
+// and to the right are single VIADDMNMX ops:  D = max(D_up - E, X_up),  I = max(I_left - E, X_left),
+// H = X_diag + sub + (O+E),  S = max3(H, D, I).  y-drop uses W = V - Y (V = best live score of the
+// rectangle [0,i]x[0,j], reading R3):  thr = max(W_up, W_left), live iff S >= thr, W = max(thr, S - Y).
+// Only S is killed (dead X = NEG); I and D keep their values -- by the lemma in DESIGN.md (V never decreases
+// along a predecessor edge) this yields the same live set, scores, peak and on-path traceback codes as
+// killing all three.  Substitution scores come from a per-column profile (4 x int16 for the column's query
+// base, streamed through a per-warp shared-memory ring) selected per row with one PRMT.
+#pragma once
+#include <cstdint>
+#include <climits>
+
+namespace fz {
+
+constexpr int NEG = -(1 << 30);   // dead score (X space)
+constexpr int BIG = (1 << 30);    // threshold of rows beyond M: nothing there is ever live
+constexpr unsigned FULL = 0xffffffffu;
+constexpr int SCORE_LIMIT = 1 << 29;
+constexpr int CP_RING = 128;      // column-profile ring entries per warp (+16 mirrored)
+constexpr int EAGER_W = 17;       // eager code window: rows/cols 0..16 (16x16)
+
+// side flags
+constexpr uint32_t SF_EAGER = 1u, SF_OVERFLOW = 2u, SF_RING = 4u, SF_EXEC_MISMATCH = 8u;
+
+struct DevParams {
+    int cp[10];        // column profile per query base b (0..3) and the zero profile (b = 4):
+                       //   cp[2b] = (sub(A,b) & 0xffff) | sub(C,b) << 16, cp[2b+1] = (sub(G,b) & 0xffff) | sub(T,b) << 16
+    int O, E, Y, OE;   // gap open, extend, y-drop, O+E
+    int K, eager_max;
+};
+
+__device__ __forceinline__ int prmt(int a, int b, int s) {
+    int d;
+    asm("prmt.b32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(s));
+    return d;
+}
+
+// PRMT selector picking the signed int16 sub(a, .) out of a column profile {lo, hi} (bytes 2a, 2a+1,
+// sign-replicated into bytes 2 and 3).
+__device__ __forceinline__ int row_selector(int a) {
+    const int b0 = 2 * a, b1 = 2 * a + 1;
+    return b0 | (b1 << 4) | ((8 | b1) << 8) | ((8 | b1) << 12);
+}
+
+// base k (0-based position pos) of a 2-bit packed sequence (16 bases per word, base 0 in bits 1:0)
+__device__ __forceinline__ int base_at(const uint32_t* __restrict__ pk, int64_t pos) {
+    return (int)((__ldg(pk + (pos >> 4)) >> ((pos & 15) * 2)) & 3u);
+}
+
+__device__ __forceinline__ int imax(int a, int b) { return a > b ? a : b; }
+
+// Traceback code of a cell (2 bits S source + 1 bit D extends + 1 bit I extends).
+//   src 0 = H (diagonal), 1 = D (up), 2 = I (left); priority H > D > I (reading R4).
+__device__ __forceinline__ uint32_t cell_code(int h, int d, int i, int du, int xu, int il, int xl, int E) {
+    uint32_t src = d > h ? 1u : 0u;
+    const int m = imax(h, d);
+    src = i > m ? 2u : src;
+    const uint32_t dext = (du - E) > xu ? 4u : 0u;
+    const uint32_t iext = (il - E) > xl ? 8u : 0u;
+    return src | dext | iext;
+}
+
+}  // namespace fz

@@ -1,0 +1,76 @@
+// internal.h -- launchers shared between kernels.cu and api.cu (not part of the ABI).
+#pragma once
+#include <cuda_runtime.h>
+#include <cstdint>
+#include "dp.cuh"
+
+namespace fz {
+
+constexpr int WARPS = 4;  // warps per block of the persistent DP kernels
+
+// Per-side arrays written by the inspector (index 2*seed + right).
+struct SideArrays {
+    int* score;          // peak score (S space)
+    int* ti;             // i*
+    int* qj;             // j*
+    uint32_t* flags;     // SF_* | eager op count << 8
+    unsigned long long* eops;  // eager ops, 2 bits each, emission order (peak -> origin)
+    long long* bound;    // executor words bound (0 for eager sides)
+};
+
+struct Batch {
+    const uint32_t *Tf, *Tr, *Qf, *Qr;  // packed target/query, forward and reversed
+    int tlen, qlen;
+    const long long* seeds;             // (tpos, qpos) pairs
+    int nseeds;
+};
+
+struct ExecPlan {
+    // per side (2n), exclusive scans in side order
+    long long* woff;     // code-word offset of the side in the pool
+    long long* soff;     // strip-table offset
+    long long* roff;     // run-buffer offset
+    int* bin;            // per side bin (0 = eager)
+    int* list;           // executor order: non-eager sides, larger bins first
+    int* counters;       // [0] inspector queue, [1] executor queue, [2..9] bin counts, [10..17] bin cursors
+    long long* totals;   // [0] words, [1] strips, [2] runs, [3] n_exec
+};
+
+struct Outputs {
+    uint32_t* codes;     // executor pool
+    int2* stab;          // strip tables
+    uint32_t* runs;      // traceback runs (len << 2 | op), emission order
+    int* nruns;          // per side
+    long long* cig_len;  // per seed CIGAR length, then exclusive-scanned in place into offsets
+    char* cigar;
+    void* recs;          // fastz_alignment[n]
+};
+
+int pick_R();  // rows per lane (FASTZ_R env: 2, 4 or 8; default 4)
+
+cudaError_t launch_pack(const char* src, int64_t n, uint32_t* fwd, uint32_t* rev, long long* bad,
+                        cudaStream_t st);
+cudaError_t launch_validate_seeds(const long long* seeds, int n, int tlen, int qlen, long long* bad,
+                                  cudaStream_t st);
+int inspector_blocks_per_sm(int R);
+cudaError_t launch_inspect(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
+                           const SideArrays& sa, int* counter, cudaStream_t st);
+cudaError_t launch_census(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
+                          long long* cells, int* counter, cudaStream_t st);
+cudaError_t launch_bin(int R, const SideArrays& sa, int nsides, const ExecPlan& pl, void* scan_tmp,
+                       size_t scan_tmp_bytes, long long* tmp_a, long long* tmp_b, long long* tmp_c,
+                       cudaStream_t st);
+size_t scan_tmp_bytes(int n);
+cudaError_t launch_execute(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
+                           const SideArrays& sa, const ExecPlan& pl, int nexec, const Outputs& o,
+                           cudaStream_t st);
+cudaError_t launch_traceback(int R, const SideArrays& sa, const ExecPlan& pl, int nexec, const Outputs& o,
+                             cudaStream_t st);
+cudaError_t launch_combine_len(const DevParams& P, const Batch& b, const SideArrays& sa, const ExecPlan& pl,
+                               const Outputs& o, void* scan_tmp, size_t scan_tmp_bytes, long long* total,
+                               cudaStream_t st);
+cudaError_t launch_combine_write(const DevParams& P, const Batch& b, const SideArrays& sa,
+                                 const ExecPlan& pl, const Outputs& o, cudaStream_t st);
+cudaError_t int_peak_run(int device, float ms, double* ops_per_s, double* mhz);
+
+}  // namespace fz

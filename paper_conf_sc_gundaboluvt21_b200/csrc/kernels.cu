@@ -1,0 +1,561 @@
+// kernels.cu -- sm_100a kernels of the FastZ hot path: pack, inspector, census, binning, executor,
+// traceback, CIGAR assembly.  Citations P:<n> are PAPER.md lines; readings R1..R8 are in DESIGN.md.
+#include <cub/device/device_scan.cuh>
+
+#include "../../include/fastz.h"
+#include "internal.h"
+#include "side.cuh"
+
+namespace fz {
+
+// ------------------------------------------------------------------------------------------------- pack
+// ASCII -> 2-bit codes (A0 C1 G2 T3, lowercase folded), forward and reversed copies (the left extension
+// reads the reversed copies).  One thread per output word of 16 bases.
+__device__ __forceinline__ int code_of(unsigned char c) {
+    switch (c) {
+        case 'A': case 'a': return 0;
+        case 'C': case 'c': return 1;
+        case 'G': case 'g': return 2;
+        case 'T': case 't': return 3;
+        default: return -1;
+    }
+}
+
+__global__ void k_pack(const char* __restrict__ src, long long n, uint32_t* __restrict__ fwd,
+                       uint32_t* __restrict__ rev, long long* bad) {
+    const long long w = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    const long long nw = (n + 15) / 16;
+    if (w >= nw) return;
+    uint32_t f = 0, r = 0;
+#pragma unroll 4
+    for (int i = 0; i < 16; ++i) {
+        const long long p = 16 * w + i;
+        if (p < n) {
+            int c = code_of((unsigned char)src[p]);
+            if (c < 0) { atomicMin(bad, p); c = 0; }
+            f |= (uint32_t)c << (2 * i);
+            int cr = code_of((unsigned char)src[n - 1 - p]);
+            if (cr < 0) cr = 0;
+            r |= (uint32_t)cr << (2 * i);
+        }
+    }
+    fwd[w] = f;
+    rev[w] = r;
+}
+
+cudaError_t launch_pack(const char* src, int64_t n, uint32_t* fwd, uint32_t* rev, long long* bad,
+                        cudaStream_t st) {
+    const long long nw = (n + 15) / 16;
+    if (nw == 0) return cudaSuccess;
+    k_pack<<<(unsigned)((nw + 255) / 256), 256, 0, st>>>(src, n, fwd, rev, bad);
+    return cudaGetLastError();
+}
+
+__global__ void k_validate_seeds(const long long* __restrict__ seeds, int n, int tlen, int qlen, long long* bad) {
+    const int s = blockIdx.x * blockDim.x + threadIdx.x;
+    if (s >= n) return;
+    const long long t = seeds[2 * s], q = seeds[2 * s + 1];
+    if (t < 0 || t > tlen || q < 0 || q > qlen) atomicMin(bad, (long long)s);
+}
+
+cudaError_t launch_validate_seeds(const long long* seeds, int n, int tlen, int qlen, long long* bad,
+                                  cudaStream_t st) {
+    if (n == 0) return cudaSuccess;
+    k_validate_seeds<<<(n + 255) / 256, 256, 0, st>>>(seeds, n, tlen, qlen, bad);
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------------- sides
+// Side 2s is seed s's left extension (A_k = T[tpos-k], B_k = Q[qpos-k]: reversed copies starting at
+// tlen - tpos, qlen - qpos), side 2s+1 its right extension (A_k = T[tpos+k-1], B_k = Q[qpos+k-1]) -- P:168.
+__device__ __forceinline__ void setup_side(const Batch& b, int side, SideIO& io) {
+    const int seed = side >> 1;
+    const long long tpos = b.seeds[2 * seed], qpos = b.seeds[2 * seed + 1];
+    if (side & 1) {
+        io.Apk = b.Tf; io.Aoff = tpos; io.M = (int)(b.tlen - tpos);
+        io.Bpk = b.Qf; io.Boff = qpos; io.Bmax = (int)(b.qlen - qpos);
+    } else {
+        io.Apk = b.Tr; io.Aoff = b.tlen - tpos; io.M = (int)tpos;
+        io.Bpk = b.Qr; io.Boff = b.qlen - qpos; io.Bmax = (int)qpos;
+    }
+    io.N = io.Bmax;
+}
+
+constexpr int OP_M = 0, OP_I = 1, OP_D = 2;
+
+struct SmemDP {
+    int2 cpr[WARPS][CP_RING + 16];
+    int2 cptab[8];
+    uint8_t ecodes[WARPS][EAGER_W * EAGER_W + 15];
+};
+
+__device__ __forceinline__ void smem_init(SmemDP& sm, const DevParams& P) {
+    if (threadIdx.x < 5) sm.cptab[threadIdx.x] = make_int2(P.cp[2 * threadIdx.x], P.cp[2 * threadIdx.x + 1]);
+    __syncthreads();
+}
+
+// ------------------------------------------------------------------------------------------------- inspector
+// Persistent: each warp pops one-sided extensions from an atomic queue (load balance replaces the paper's
+// 32 CUDA streams).  Score-only DP + eager 17x17 corner codes; when the peak lies inside the
+// eager window the warp's lane 0 walks the codes at once and the side skips the executor.
+template <int R>
+__global__ void __launch_bounds__(WARPS * 32) k_inspect(DevParams P, Batch b, int4* ring, int rmask,
+                                                         SideArrays sa, int* counter) {
+    __shared__ SmemDP sm;
+    smem_init(sm, P);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    SideIO io;
+    io.ring = ring + (size_t)(blockIdx.x * WARPS + warp) * (size_t)(rmask + 1);
+    io.rmask = rmask;
+    io.cpring = sm.cpr[warp];
+    io.cptab = sm.cptab;
+    io.ecodes = sm.ecodes[warp];
+    io.eager_max = P.eager_max;
+    io.codes = nullptr;
+    io.stab = nullptr;
+    const int nsides = 2 * b.nseeds;
+    for (;;) {
+        int side = 0;
+        if (lane == 0) side = atomicAdd(counter, 1);
+        side = __shfl_sync(FULL, side, 0);
+        if (side >= nsides) break;
+        setup_side(b, side, io);
+        SideOut o;
+        run_side<R, MODE_INSPECT, true>(P, io, o);
+        __syncwarp();  // eager corner codes (shared memory) written by lanes 0..4 -> read by lane 0
+        if (lane == 0) {
+            uint32_t flags = o.flags;
+            unsigned long long ops = 0;
+            int nops = 0;
+            const bool eager = o.bi <= P.eager_max && o.bj <= P.eager_max && !(flags & (SF_RING | SF_OVERFLOW));
+            if (eager) {
+                int i = o.bi, j = o.bj, state = 0;
+                while (i > 0 || j > 0) {
+                    const uint32_t code = io.ecodes[i * EAGER_W + j];
+                    if (state == 0) {
+                        const uint32_t src = code & 3u;
+                        if (src == 0) {
+                            ops |= (unsigned long long)OP_M << (2 * nops);
+                            ++nops; --i; --j;
+                            continue;
+                        }
+                        state = (int)src;
+                    }
+                    if (state == 1) {
+                        ops |= (unsigned long long)OP_D << (2 * nops);
+                        ++nops;
+                        state = (code >> 2) & 1u ? 1 : 0;
+                        --i;
+                    } else {
+                        ops |= (unsigned long long)OP_I << (2 * nops);
+                        ++nops;
+                        state = (code >> 3) & 1u ? 2 : 0;
+                        --j;
+                    }
+                }
+                flags |= SF_EAGER;
+            }
+            sa.score[side] = o.best + P.OE;
+            sa.ti[side] = o.bi;
+            sa.qj[side] = o.bj;
+            sa.flags[side] = flags | ((uint32_t)nops << 8);
+            sa.eops[side] = ops;
+            sa.bound[side] = eager ? 0 : o.bound_words;
+        }
+        __syncwarp();
+    }
+}
+
+template <int R>
+__global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int4* ring, int rmask,
+                                                        long long* cells, int* counter) {
+    __shared__ SmemDP sm;
+    smem_init(sm, P);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    SideIO io;
+    io.ring = ring + (size_t)(blockIdx.x * WARPS + warp) * (size_t)(rmask + 1);
+    io.rmask = rmask;
+    io.cpring = sm.cpr[warp];
+    io.cptab = sm.cptab;
+    io.ecodes = nullptr;
+    io.eager_max = -1;
+    io.codes = nullptr;
+    io.stab = nullptr;
+    const int nsides = 2 * b.nseeds;
+    for (;;) {
+        int side = 0;
+        if (lane == 0) side = atomicAdd(counter, 1);
+        side = __shfl_sync(FULL, side, 0);
+        if (side >= nsides) break;
+        setup_side(b, side, io);
+        SideOut o;
+        run_side<R, MODE_CENSUS, false>(P, io, o);
+        if (lane == 0) cells[side] = (o.flags & SF_RING) ? -1 : o.cells;
+        __syncwarp();
+    }
+}
+
+// ------------------------------------------------------------------------------------------------- executor
+// Trimmed executor: the DP over [0,i*]x[0,j*] only, writing traceback codes.  Persistent warps
+// pop non-eager sides in bin order, largest bins first (length binning P:209-211 used as an LPT schedule).
+template <int R>
+__global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, int4* ring, int rmask,
+                                                         SideArrays sa, ExecPlan pl, int nexec, Outputs out) {
+    __shared__ SmemDP sm;
+    smem_init(sm, P);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    SideIO io;
+    io.ring = ring + (size_t)(blockIdx.x * WARPS + warp) * (size_t)(rmask + 1);
+    io.rmask = rmask;
+    io.cpring = sm.cpr[warp];
+    io.cptab = sm.cptab;
+    io.ecodes = nullptr;
+    io.eager_max = -1;
+    for (;;) {
+        int idx = 0;
+        if (lane == 0) idx = atomicAdd(&pl.counters[1], 1);
+        idx = __shfl_sync(FULL, idx, 0);
+        if (idx >= nexec) break;
+        const int side = pl.list[idx];
+        setup_side(b, side, io);
+        io.M = sa.ti[side];
+        io.N = sa.qj[side];
+        io.codes = out.codes + pl.woff[side];
+        io.stab = out.stab + pl.soff[side];
+        SideOut o;
+        run_side<R, MODE_EXEC, false>(P, io, o);
+        if (lane == 0 && (o.flags & SF_RING)) atomicOr(&sa.flags[side], SF_RING);
+        __syncwarp();
+    }
+}
+
+// ------------------------------------------------------------------------------------------------- traceback
+// One thread per executed side (inter-seed traceback parallelism).  Walks the 4-bit codes from
+// (i*, j*) in state S to the origin; emits run-length ops (len << 2 | op) in peak -> origin order.
+template <int R>
+__global__ void k_traceback(SideArrays sa, ExecPlan pl, int nexec, Outputs out) {
+    constexpr int H = 32 * R, SPW = 8 / R;
+    const int idx = blockIdx.x * blockDim.x + threadIdx.x;
+    if (idx >= nexec) return;
+    const int side = pl.list[idx];
+    const uint32_t* __restrict__ codes = out.codes + pl.woff[side];
+    const int2* __restrict__ stab = out.stab + pl.soff[side];
+    uint32_t* __restrict__ runs = out.runs + pl.roff[side];
+    int i = sa.ti[side], j = sa.qj[side], state = 0, nr = 0;
+    uint32_t cur = 0xffffffffu, len = 0;
+    auto emit = [&](uint32_t op) {
+        if (op == cur) {
+            ++len;
+        } else {
+            if (len) runs[nr++] = (len << 2) | cur;
+            cur = op;
+            len = 1;
+        }
+    };
+    while (i > 0 || j > 0) {
+        const int s = i / H, lr = i - s * H, ln = lr / R, k = lr - ln * R;
+        const int2 st = stab[s];
+        const int t = j - st.x + ln;
+        const uint32_t w = codes[(long long)st.y + (long long)(t / SPW) * 32 + ln];
+        const uint32_t code = (w >> ((((t % SPW) * R) + k) * 4)) & 15u;
+        if (state == 0) {
+            const uint32_t src = code & 3u;
+            if (src == 0) {
+                emit(OP_M);
+                --i; --j;
+                continue;
+            }
+            state = (int)src;
+        }
+        if (state == 1) {
+            emit(OP_D);
+            state = (code >> 2) & 1u ? 1 : 0;
+            --i;
+        } else {
+            emit(OP_I);
+            state = (code >> 3) & 1u ? 2 : 0;
+            --j;
+        }
+    }
+    if (len) runs[nr++] = (len << 2) | cur;
+    out.nruns[side] = nr;
+}
+
+// ------------------------------------------------------------------------------------------------- binning
+// Bins by max(i*, j*) (512, 2048, 8192, 32768, then 4x): bin 0 = eager.
+__device__ __forceinline__ int bin_of(int m) {
+    if (m <= 512) return 1;
+    if (m <= 2048) return 2;
+    if (m <= 8192) return 3;
+    if (m <= 32768) return 4;
+    if (m <= 131072) return 5;
+    return 6;
+}
+
+template <int R>
+__global__ void k_bin_count(SideArrays sa, int nsides, ExecPlan pl, long long* words, long long* strips,
+                            long long* runs) {
+    const int s = blockIdx.x * blockDim.x + threadIdx.x;
+    if (s >= nsides) return;
+    const bool eager = sa.flags[s] & SF_EAGER;
+    const int ti = sa.ti[s], qj = sa.qj[s];
+    const int bin = eager ? 0 : bin_of(ti > qj ? ti : qj);
+    pl.bin[s] = bin;
+    atomicAdd(&pl.counters[2 + bin], 1);
+    if (sa.flags[s] & SF_RING) atomicOr(&pl.counters[20], 1);
+    words[s] = eager ? 0 : sa.bound[s];
+    strips[s] = eager ? 0 : ti / (32 * R) + 1;
+    runs[s] = eager ? 0 : (long long)ti + qj + 1;
+}
+
+__global__ void k_bin_offsets(ExecPlan pl, int nsides, const long long* words, const long long* strips,
+                              const long long* runs) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    int run = 0;
+    for (int bin = 6; bin >= 1; --bin) {  // larger bins first
+        pl.counters[10 + bin] = run;
+        run += pl.counters[2 + bin];
+    }
+    if (nsides > 0) {
+        pl.totals[0] = pl.woff[nsides - 1] + words[nsides - 1];
+        pl.totals[1] = pl.soff[nsides - 1] + strips[nsides - 1];
+        pl.totals[2] = pl.roff[nsides - 1] + runs[nsides - 1];
+    } else {
+        pl.totals[0] = pl.totals[1] = pl.totals[2] = 0;
+    }
+    pl.totals[3] = run;
+}
+
+__global__ void k_bin_scatter(ExecPlan pl, int nsides) {
+    const int s = blockIdx.x * blockDim.x + threadIdx.x;
+    if (s >= nsides) return;
+    const int bin = pl.bin[s];
+    if (bin == 0) return;
+    const int pos = atomicAdd(&pl.counters[10 + bin], 1);
+    pl.list[pos] = s;
+}
+
+size_t scan_tmp_bytes(int n) {
+    size_t bytes = 0;
+    cub::DeviceScan::ExclusiveSum(nullptr, bytes, (const long long*)nullptr, (long long*)nullptr, n > 0 ? n : 1);
+    return bytes;
+}
+
+cudaError_t launch_bin(int R, const SideArrays& sa, int nsides, const ExecPlan& pl, void* tmp, size_t tmp_bytes,
+                       long long* words, long long* strips, long long* runs, cudaStream_t st) {
+    if (nsides > 0) {
+        const int g = (nsides + 255) / 256;
+        switch (R) {
+            case 2: k_bin_count<2><<<g, 256, 0, st>>>(sa, nsides, pl, words, strips, runs); break;
+            case 8: k_bin_count<8><<<g, 256, 0, st>>>(sa, nsides, pl, words, strips, runs); break;
+            default: k_bin_count<4><<<g, 256, 0, st>>>(sa, nsides, pl, words, strips, runs); break;
+        }
+        cudaError_t e;
+        size_t b = tmp_bytes;
+        if ((e = cub::DeviceScan::ExclusiveSum(tmp, b, words, pl.woff, nsides, st)) != cudaSuccess) return e;
+        b = tmp_bytes;
+        if ((e = cub::DeviceScan::ExclusiveSum(tmp, b, strips, pl.soff, nsides, st)) != cudaSuccess) return e;
+        b = tmp_bytes;
+        if ((e = cub::DeviceScan::ExclusiveSum(tmp, b, runs, pl.roff, nsides, st)) != cudaSuccess) return e;
+    }
+    k_bin_offsets<<<1, 1, 0, st>>>(pl, nsides, words, strips, runs);
+    if (nsides > 0) k_bin_scatter<<<(nsides + 255) / 256, 256, 0, st>>>(pl, nsides);
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------------- combine
+// Seed s = left side 2s (ops emitted peak -> origin in the reversed frame == forward order) followed by the
+// right side 2s+1 (emitted peak -> origin == backward, so read in reverse); equal neighbours merge.
+struct RunVisitor {
+    const SideArrays& sa;
+    const ExecPlan& pl;
+    const Outputs& o;
+    template <class F>
+    __device__ __forceinline__ void visit(int seed, F&& f) const {
+        const int L = 2 * seed, Rt = 2 * seed + 1;
+        uint32_t cur = 0xffffffffu;
+        long long len = 0;
+        auto push = [&](uint32_t op, long long n) {
+            if (op == cur) {
+                len += n;
+            } else {
+                if (len) f(cur, len);
+                cur = op;
+                len = n;
+            }
+        };
+        {
+            const uint32_t fl = sa.flags[L];
+            if (fl & SF_EAGER) {
+                const int n = (fl >> 8) & 0xff;
+                const unsigned long long ops = sa.eops[L];
+                for (int k = 0; k < n; ++k) push((uint32_t)(ops >> (2 * k)) & 3u, 1);
+            } else {
+                const uint32_t* r = o.runs + pl.roff[L];
+                const int n = o.nruns[L];
+                for (int k = 0; k < n; ++k) push(r[k] & 3u, r[k] >> 2);
+            }
+        }
+        {
+            const uint32_t fl = sa.flags[Rt];
+            if (fl & SF_EAGER) {
+                const int n = (fl >> 8) & 0xff;
+                const unsigned long long ops = sa.eops[Rt];
+                for (int k = n - 1; k >= 0; --k) push((uint32_t)(ops >> (2 * k)) & 3u, 1);
+            } else {
+                const uint32_t* r = o.runs + pl.roff[Rt];
+                const int n = o.nruns[Rt];
+                for (int k = n - 1; k >= 0; --k) push(r[k] & 3u, r[k] >> 2);
+            }
+        }
+        if (len) f(cur, len);
+    }
+};
+
+__device__ __forceinline__ int ndigits(long long v) {
+    int d = 1;
+    while (v >= 10) { v /= 10; ++d; }
+    return d;
+}
+
+__global__ void k_combine_len(Batch b, SideArrays sa, ExecPlan pl, Outputs o, long long* lens) {
+    const int s = blockIdx.x * blockDim.x + threadIdx.x;
+    if (s >= b.nseeds) return;
+    RunVisitor v{sa, pl, o};
+    long long n = 0;
+    v.visit(s, [&](uint32_t, long long len) { n += ndigits(len) + 1; });
+    lens[s] = n;
+}
+
+__global__ void k_combine_total(const long long* offs, const long long* lens, int n, long long* total) {
+    if (threadIdx.x == 0 && blockIdx.x == 0) *total = n > 0 ? offs[n - 1] + lens[n - 1] : 0;
+}
+
+cudaError_t launch_combine_len(const DevParams&, const Batch& b, const SideArrays& sa, const ExecPlan& pl,
+                               const Outputs& o, void* tmp, size_t tmp_bytes, long long* total, cudaStream_t st) {
+    const int n = b.nseeds;  // o.cig_len holds 2n entries: offsets [0, n), lengths [n, 2n)
+    if (n > 0) {
+        k_combine_len<<<(n + 255) / 256, 256, 0, st>>>(b, sa, pl, o, o.cig_len + n);
+        size_t bb = tmp_bytes;
+        cudaError_t e = cub::DeviceScan::ExclusiveSum(tmp, bb, o.cig_len + n, o.cig_len, n, st);
+        if (e != cudaSuccess) return e;
+    }
+    k_combine_total<<<1, 1, 0, st>>>(o.cig_len, o.cig_len + n, n, total);
+    return cudaGetLastError();
+}
+
+__global__ void k_combine_write(DevParams P, Batch b, SideArrays sa, ExecPlan pl, Outputs o) {
+    const int s = blockIdx.x * blockDim.x + threadIdx.x;
+    if (s >= b.nseeds) return;
+    RunVisitor v{sa, pl, o};
+    const long long off = o.cig_len[s];
+    char* out = o.cigar + off;
+    long long n = 0;
+    v.visit(s, [&](uint32_t op, long long len) {
+        const int d = ndigits(len);
+        for (int k = d - 1; k >= 0; --k) {
+            out[n + k] = (char)('0' + len % 10);
+            len /= 10;
+        }
+        n += d;
+        out[n++] = op == OP_M ? 'M' : (op == OP_I ? 'I' : 'D');
+    });
+    const int L = 2 * s, Rt = 2 * s + 1;
+    const long long tpos = b.seeds[2 * s], qpos = b.seeds[2 * s + 1];
+    fastz_alignment a;
+    a.left_score = sa.score[L];
+    a.right_score = sa.score[Rt];
+    a.score = a.left_score + a.right_score;
+    const uint32_t fl = sa.flags[L], fr = sa.flags[Rt];
+    a.flags = (a.score >= P.K ? FASTZ_FLAG_ABOVE_K : 0u) | ((fl & SF_EAGER) ? FASTZ_FLAG_LEFT_EAGER : 0u) |
+              ((fr & SF_EAGER) ? FASTZ_FLAG_RIGHT_EAGER : 0u) |
+              (((fl | fr) & SF_OVERFLOW) ? FASTZ_FLAG_OVERFLOW : 0u);
+    a.t_start = tpos - sa.ti[L];
+    a.t_end = tpos + sa.ti[Rt];
+    a.q_start = qpos - sa.qj[L];
+    a.q_end = qpos + sa.qj[Rt];
+    a.cigar_off = off;
+    a.cigar_len = (int32_t)n;
+    a.reserved = 0;
+    reinterpret_cast<fastz_alignment*>(o.recs)[s] = a;
+}
+
+cudaError_t launch_combine_write(const DevParams& P, const Batch& b, const SideArrays& sa, const ExecPlan& pl,
+                                 const Outputs& o, cudaStream_t st) {
+    if (b.nseeds == 0) return cudaSuccess;
+    k_combine_write<<<(b.nseeds + 127) / 128, 128, 0, st>>>(P, b, sa, pl, o);
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------------- launchers
+int pick_R() {
+    static int r = 0;
+    if (!r) {
+        const char* e = getenv("FASTZ_R");
+        r = e ? atoi(e) : 4;
+        if (r != 2 && r != 4 && r != 8) r = 4;
+    }
+    return r;
+}
+
+template <int R>
+static int bps_of() {
+    int n = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_inspect<R>, WARPS * 32, 0);
+    return n > 0 ? n : 1;
+}
+
+int inspector_blocks_per_sm(int R) {
+    switch (R) {
+        case 2: return bps_of<2>();
+        case 8: return bps_of<8>();
+        default: return bps_of<4>();
+    }
+}
+
+cudaError_t launch_inspect(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
+                           const SideArrays& sa, int* counter, cudaStream_t st) {
+    if (b.nseeds == 0) return cudaSuccess;
+    switch (R) {
+        case 2: k_inspect<2><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, counter); break;
+        case 8: k_inspect<8><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, counter); break;
+        default: k_inspect<4><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, counter); break;
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t launch_census(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
+                          long long* cells, int* counter, cudaStream_t st) {
+    if (b.nseeds == 0) return cudaSuccess;
+    switch (R) {
+        case 2: k_census<2><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, cells, counter); break;
+        case 8: k_census<8><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, cells, counter); break;
+        default: k_census<4><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, cells, counter); break;
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t launch_execute(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
+                           const SideArrays& sa, const ExecPlan& pl, int nexec, const Outputs& o, cudaStream_t st) {
+    if (nexec == 0) return cudaSuccess;
+    switch (R) {
+        case 2: k_execute<2><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, pl, nexec, o); break;
+        case 8: k_execute<8><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, pl, nexec, o); break;
+        default: k_execute<4><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, pl, nexec, o); break;
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t launch_traceback(int R, const SideArrays& sa, const ExecPlan& pl, int nexec, const Outputs& o,
+                             cudaStream_t st) {
+    if (nexec == 0) return cudaSuccess;
+    const int g = (nexec + 127) / 128;
+    switch (R) {
+        case 2: k_traceback<2><<<g, 128, 0, st>>>(sa, pl, nexec, o); break;
+        case 8: k_traceback<8><<<g, 128, 0, st>>>(sa, pl, nexec, o); break;
+        default: k_traceback<4><<<g, 128, 0, st>>>(sa, pl, nexec, o); break;
+    }
+    return cudaGetLastError();
+}
+
+}  // namespace fz

@@ -1,0 +1,264 @@
+"""Thin ctypes binding of libfastz.so (include/fastz.h).  Argument marshalling only: every step of the
+hot path runs in the library's CUDA kernels.  There is no CPU fallback -- if libfastz.so is missing or no
+CUDA device is present, the calls fail loudly.
+
+Function names mirror the C ABI (fastz_create, fastz_extend_seeds, fastz_get_alignments, ...); the
+:class:`Aligner` class wraps them for convenience.  PyTorch is used only to hand over device memory and
+the current CUDA stream when the caller passes torch tensors.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass, field
+
+import numpy as np
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "libfastz.so")
+
+FASTZ_OK, FASTZ_EINVAL, FASTZ_EBASE, FASTZ_ERANGE = 0, -1, -2, -3
+FASTZ_ENOMEM, FASTZ_ECUDA, FASTZ_ETRUNC, FASTZ_ESTATE = -4, -5, -6, -7
+FLAG_ABOVE_K, FLAG_LEFT_EAGER, FLAG_RIGHT_EAGER, FLAG_OVERFLOW = 1, 2, 4, 8
+
+# names declared in include/fastz.h (checked by tests/test_abi.py against the header)
+EXPORTS = ["fastz_default_params", "fastz_create", "fastz_extend_seeds", "fastz_get_alignments",
+           "fastz_get_alignments_device", "fastz_get_sides", "fastz_census", "fastz_get_stats",
+           "fastz_destroy", "fastz_strerror", "fastz_int_peak"]
+
+
+class FastzError(RuntimeError):
+    def __init__(self, status: int, text: str):
+        super().__init__(f"fastz status {status}: {text}")
+        self.status = status
+
+
+class fastz_params(ctypes.Structure):
+    _fields_ = [("sub", ctypes.c_int32 * 16), ("gap_open", ctypes.c_int32), ("gap_extend", ctypes.c_int32),
+                ("ydrop", ctypes.c_int32), ("gapped_threshold", ctypes.c_int32), ("eager_max", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 3), ("dev_alloc", ctypes.c_void_p), ("dev_free", ctypes.c_void_p),
+                ("alloc_user", ctypes.c_void_p)]
+
+
+class fastz_stats(ctypes.Structure):
+    _fields_ = [("ms_total", ctypes.c_float), ("ms_upload", ctypes.c_float), ("ms_inspect", ctypes.c_float),
+                ("ms_bin", ctypes.c_float), ("ms_execute", ctypes.c_float), ("ms_traceback", ctypes.c_float),
+                ("ms_combine", ctypes.c_float), ("n_warp_slots", ctypes.c_int32), ("n_seeds", ctypes.c_int64),
+                ("n_sides", ctypes.c_int64), ("n_eager_sides", ctypes.c_int64), ("n_exec_sides", ctypes.c_int64),
+                ("bin_counts", ctypes.c_int64 * 8), ("exec_words", ctypes.c_int64), ("cigar_bytes", ctypes.c_int64)]
+
+
+ALIGN_DTYPE = np.dtype([("score", "<i4"), ("left_score", "<i4"), ("right_score", "<i4"), ("flags", "<u4"),
+                        ("t_start", "<i8"), ("t_end", "<i8"), ("q_start", "<i8"), ("q_end", "<i8"),
+                        ("cigar_off", "<i8"), ("cigar_len", "<i4"), ("reserved", "<i4")])
+assert ALIGN_DTYPE.itemsize == 64
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    """Load libfastz.so; raises if it has not been built (no fallback path exists)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: build it with `python -m paper_conf_sc_gundaboluvt21_b200.build` "
+                          "(there is no CPU fallback)")
+    L = ctypes.CDLL(LIB_PATH)
+    vp, i64, i32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int
+    L.fastz_default_params.argtypes = [ctypes.POINTER(fastz_params)]
+    L.fastz_default_params.restype = None
+    L.fastz_create.argtypes = [ctypes.POINTER(fastz_params), vp, i64, vp, i64, i32, vp, ctypes.POINTER(vp)]
+    L.fastz_extend_seeds.argtypes = [vp, vp, i64, i32]
+    L.fastz_get_alignments.argtypes = [vp, vp, i64, vp, i64, ctypes.POINTER(i64), ctypes.POINTER(i64)]
+    L.fastz_get_alignments_device.argtypes = [vp, ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.POINTER(i64),
+                                              ctypes.POINTER(i64)]
+    L.fastz_get_sides.argtypes = [vp, vp, vp, vp, vp, i64]
+    L.fastz_census.argtypes = [vp, vp, i64]
+    L.fastz_get_stats.argtypes = [vp, ctypes.POINTER(fastz_stats)]
+    L.fastz_destroy.argtypes = [vp]
+    L.fastz_destroy.restype = None
+    L.fastz_strerror.argtypes = [i32]
+    L.fastz_strerror.restype = ctypes.c_char_p
+    L.fastz_int_peak.argtypes = [i32, ctypes.c_float, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)]
+    for name in ("fastz_create", "fastz_extend_seeds", "fastz_get_alignments", "fastz_get_alignments_device",
+                 "fastz_get_sides", "fastz_census", "fastz_get_stats", "fastz_int_peak"):
+        getattr(L, name).restype = i32
+    _lib = L
+    return L
+
+
+def _check(status: int):
+    if status != FASTZ_OK:
+        raise FastzError(status, lib().fastz_strerror(status).decode())
+
+
+# ----------------------------------------------------------------------------------- C-named wrappers
+
+def fastz_default_params(**overrides) -> fastz_params:
+    p = fastz_params()
+    lib().fastz_default_params(ctypes.byref(p))
+    for k, v in overrides.items():
+        if k == "sub":
+            flat = np.asarray(v, dtype=np.int32).reshape(16)
+            for i in range(16):
+                p.sub[i] = int(flat[i])
+        else:
+            setattr(p, k, int(v))
+    return p
+
+
+def _ptr_len(x):
+    """(pointer, length, is_device) for bytes / numpy / torch inputs."""
+    try:
+        import torch
+        if isinstance(x, torch.Tensor):
+            x = x.contiguous()
+            return x.data_ptr(), x.numel() * x.element_size(), x.is_cuda, x
+    except ImportError:  # pragma: no cover
+        pass
+    if isinstance(x, str):
+        x = x.encode()
+    if isinstance(x, (bytes, bytearray)):
+        buf = ctypes.create_string_buffer(bytes(x), len(x))
+        return ctypes.addressof(buf), len(x), False, buf
+    arr = np.ascontiguousarray(x)
+    return arr.ctypes.data, arr.nbytes, False, arr
+
+
+def fastz_create(params: fastz_params, target, query, device: int = 0, stream: int | None = None) -> int:
+    tp, tl, _, tk = _ptr_len(target)
+    qp, ql, _, qk = _ptr_len(query)
+    out = ctypes.c_void_p()
+    _check(lib().fastz_create(ctypes.byref(params), tp, tl, qp, ql, device, stream, ctypes.byref(out)))
+    del tk, qk
+    return out.value
+
+
+def fastz_extend_seeds(ctx: int, seeds) -> int:
+    """seeds: (n, 2) int64 cut points as numpy (host) or a CUDA torch tensor (device)."""
+    try:
+        import torch
+        if isinstance(seeds, torch.Tensor):
+            s = seeds.to(torch.int64).contiguous()
+            _check(lib().fastz_extend_seeds(ctx, s.data_ptr(), s.shape[0], 1 if s.is_cuda else 0))
+            return s.shape[0]
+    except ImportError:  # pragma: no cover
+        pass
+    s = np.ascontiguousarray(np.asarray(seeds, dtype=np.int64).reshape(-1, 2))
+    _check(lib().fastz_extend_seeds(ctx, s.ctypes.data, s.shape[0], 0))
+    return s.shape[0]
+
+
+def fastz_get_alignments(ctx: int):
+    n, nb = ctypes.c_int64(), ctypes.c_int64()
+    st = lib().fastz_get_alignments(ctx, None, 0, None, 0, ctypes.byref(n), ctypes.byref(nb))
+    if st not in (FASTZ_OK, FASTZ_ETRUNC):
+        _check(st)
+    rec = np.zeros(max(n.value, 1), dtype=ALIGN_DTYPE)
+    cig = ctypes.create_string_buffer(max(nb.value, 1))
+    _check(lib().fastz_get_alignments(ctx, rec.ctypes.data, n.value, cig, nb.value, ctypes.byref(n), ctypes.byref(nb)))
+    return rec[:n.value], cig.raw[:nb.value]
+
+
+def fastz_get_sides(ctx: int, n: int):
+    score = np.zeros(max(2 * n, 1), np.int32)
+    ti = np.zeros_like(score)
+    qj = np.zeros_like(score)
+    fl = np.zeros(max(2 * n, 1), np.uint32)
+    _check(lib().fastz_get_sides(ctx, score.ctypes.data, ti.ctypes.data, qj.ctypes.data, fl.ctypes.data, 2 * n))
+    return score[:2 * n], ti[:2 * n], qj[:2 * n], fl[:2 * n]
+
+
+def fastz_census(ctx: int, n: int) -> np.ndarray:
+    cells = np.zeros(max(2 * n, 1), np.int64)
+    _check(lib().fastz_census(ctx, cells.ctypes.data, 2 * n))
+    return cells[:2 * n]
+
+
+def fastz_get_stats(ctx: int) -> dict:
+    s = fastz_stats()
+    _check(lib().fastz_get_stats(ctx, ctypes.byref(s)))
+    d = {k: getattr(s, k) for k, _ in fastz_stats._fields_}
+    d["bin_counts"] = list(s.bin_counts)
+    return d
+
+
+def fastz_destroy(ctx: int):
+    if ctx:
+        lib().fastz_destroy(ctx)
+
+
+def fastz_int_peak(device: int = 0, ms: float = 200.0):
+    ops, mhz = ctypes.c_double(), ctypes.c_double()
+    _check(lib().fastz_int_peak(device, ms, ctypes.byref(ops), ctypes.byref(mhz)))
+    return ops.value, mhz.value
+
+
+# ----------------------------------------------------------------------------------- convenience class
+
+@dataclass
+class Alignments:
+    rec: np.ndarray
+    cigar: bytes = field(repr=False)
+
+    def cigar_of(self, s: int) -> str:
+        r = self.rec[s]
+        return self.cigar[r["cigar_off"]: r["cigar_off"] + r["cigar_len"]].decode()
+
+
+class Aligner:
+    """One context (device + stream + packed sequences).  ``extend`` returns host results; ``extend_only``
+    leaves them on the device (for timing / NCCL gathers)."""
+
+    def __init__(self, target, query, params: fastz_params | None = None, device: int = 0, stream=None, **kw):
+        self.params = params if params is not None else fastz_default_params(**kw)
+        if stream is None:
+            try:
+                import torch
+                if torch.cuda.is_available():
+                    torch.cuda.set_device(device)
+                    stream = torch.cuda.current_stream(device).cuda_stream
+            except ImportError:  # pragma: no cover
+                stream = None
+        self.ctx = fastz_create(self.params, target, query, device, stream)
+        self.n = 0
+
+    def extend_only(self, seeds) -> int:
+        self.n = fastz_extend_seeds(self.ctx, seeds)
+        return self.n
+
+    def extend(self, seeds) -> Alignments:
+        self.extend_only(seeds)
+        rec, cig = fastz_get_alignments(self.ctx)
+        return Alignments(rec, cig)
+
+    def results(self) -> Alignments:
+        rec, cig = fastz_get_alignments(self.ctx)
+        return Alignments(rec, cig)
+
+    def sides(self):
+        return fastz_get_sides(self.ctx, self.n)
+
+    def census(self) -> np.ndarray:
+        return fastz_census(self.ctx, self.n)
+
+    def stats(self) -> dict:
+        return fastz_get_stats(self.ctx)
+
+    def close(self):
+        fastz_destroy(self.ctx)
+        self.ctx = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def __del__(self):
+        try:
+            if self.ctx:
+                self.close()
+        except Exception:
+            pass

@@ -1,0 +1,144 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element by element, bit-exact
+(all arithmetic is integer).  Compared per seed: score, left/right scores, endpoints, flags, CIGAR; per
+side: peak (score, i*, j*); and the explored-cell census (the GCUPS numerator) against the oracle's count.
+"""
+import json
+import os
+import random
+
+import numpy as np
+import pytest
+
+from synth import genome
+from tests.gpu_util import compare, run_both
+
+pytestmark = pytest.mark.gpu
+HERE = os.path.dirname(os.path.abspath(__file__))
+GOLD = json.load(open(os.path.join(HERE, "golden", "worked_examples.json")))
+BASES = "ACGT"
+
+
+def rseq(rng, n):
+    return "".join(rng.choice(BASES) for _ in range(n))
+
+
+def mutate(rng, s, sub=0.1, indel=0.02):
+    out = []
+    for ch in s:
+        r = rng.random()
+        if r < indel / 2:
+            continue
+        if r < indel:
+            out.append(rng.choice(BASES))
+        out.append(rng.choice([b for b in BASES if b != ch]) if rng.random() < sub else ch)
+    return "".join(out)
+
+
+def assert_ok(bad):
+    assert not bad, bad
+
+
+@pytest.mark.parametrize("ex", GOLD["two_sided"], ids=lambda e: e["id"])
+def test_worked_two_sided(ex):
+    bad, g, o, _ = compare(ex["T"], ex["Q"], [(ex["tpos"], ex["qpos"])])
+    assert_ok(bad)
+    assert g.cigar_of(0) == ex["cigar"] and int(g.rec[0]["score"]) == ex["score"]
+
+
+@pytest.mark.parametrize("ex", GOLD["one_sided"], ids=lambda e: e["id"])
+def test_worked_one_sided_as_right_side(ex):
+    kw = {"ydrop": ex["ydrop"]} if "ydrop" in ex else {}
+    bad, g, o, _ = compare(ex["A"], ex["B"], [(0, 0)], **kw)
+    assert_ok(bad)
+    assert int(g.rec[0]["right_score"]) == ex["score"]
+
+
+def test_small_mixed_workloads():
+    for seed in range(4):
+        w = genome.small_pair(seed, length=20000, n_seeds=200)
+        bad, *_ = compare(w.T, w.Q, w.seeds)
+        assert_ok(bad)
+
+
+def test_edges_empty_sides_and_sequence_ends():
+    rng = random.Random(5)
+    T = rseq(rng, 3000)
+    Q = mutate(rng, T)
+    seeds = [(0, 0), (len(T), len(Q)), (0, len(Q)), (len(T), 0), (1, 1), (len(T) - 1, len(Q) - 1),
+             (1500, 1500), (1500, 0), (0, 1500)]
+    bad, *_ = compare(T, Q, seeds)
+    assert_ok(bad)
+
+
+def test_empty_batch_and_tiny_sequences():
+    g, sides, cells, stats, o = run_both("A", "C", np.zeros((0, 2), np.int64))
+    assert len(g.rec) == 0 and g.cigar == b""
+    bad, *_ = compare("A", "A", [(0, 0), (1, 1), (0, 1), (1, 0)])
+    assert_ok(bad)
+
+
+@pytest.mark.parametrize("Y", [0, 1, 300, 9400, 10 ** 6])
+def test_ydrop_values(Y):
+    rng = random.Random(Y)
+    T = rseq(rng, 4000)
+    Q = mutate(rng, T, sub=0.15)
+    seeds = [(rng.randint(0, 4000), rng.randint(0, len(Q))) for _ in range(40)] + \
+            [(k, k) for k in range(100, 4000, 400)]
+    bad, *_ = compare(T, Q, seeds, ydrop=Y)
+    assert_ok(bad)
+
+
+@pytest.mark.parametrize("O,E", [(0, 30), (400, 1), (50, 200), (0, 1)])
+def test_gap_parameters(O, E):
+    rng = random.Random(O * 1000 + E)
+    T = rseq(rng, 3000)
+    Q = mutate(rng, T, sub=0.1, indel=0.05)
+    seeds = [(k, min(k, len(Q))) for k in range(0, 3000, 150)]
+    bad, *_ = compare(T, Q, seeds, gap_open=O, gap_extend=E, ydrop=min(9400, O + 300 * E))
+    assert_ok(bad)
+
+
+def test_random_scoring_matrices():
+    rng = random.Random(77)
+    for trial in range(6):
+        sub = [[rng.randint(-150, 120) for _ in range(4)] for _ in range(4)]
+        T = rseq(rng, 1500)
+        Q = mutate(rng, T, sub=0.2)
+        seeds = [(rng.randint(0, 1500), rng.randint(0, len(Q))) for _ in range(30)]
+        bad, *_ = compare(T, Q, seeds, sub=sub, gap_open=rng.choice([0, 100, 400]),
+                          gap_extend=rng.choice([5, 30]), ydrop=rng.choice([200, 1000, 9400]))
+        assert_ok(bad)
+
+
+@pytest.mark.parametrize("kind", ["homopolymer", "tandem", "dinuc"])
+def test_adversarial_wide_bands(kind):
+    if kind == "homopolymer":
+        T, Q = "A" * 3000, "A" * 2500
+    elif kind == "tandem":
+        T, Q = "ACGTTG" * 500, "ACGTTG" * 450 + "ACG"
+    else:
+        T, Q = "AT" * 1500, "TA" * 1400
+    seeds = [(0, 0), (1000, 1000), (1500, 900), (len(T), len(Q)), (2000, 2400)]
+    bad, *_ = compare(T, Q, seeds)
+    assert_ok(bad)
+
+
+def test_long_homologous_multi_strip():
+    """Alignments spanning many strips (strip height 32*R rows) and long executor traceback."""
+    rng = random.Random(9)
+    T = rseq(rng, 12000)
+    Q = mutate(rng, T, sub=0.08, indel=0.01)
+    seeds = [(6000, int(len(Q) * 0.5)), (0, 0), (12000, len(Q))]
+    # exact 12-mer seeds on the diagonal
+    w = genome.config1(n_seeds=64)
+    bad, *_ = compare(T, Q, seeds)
+    assert_ok(bad)
+    bad, *_ = compare(w.T, w.Q, w.seeds[:16], census=False)
+    assert_ok(bad)
+
+
+def test_deterministic_repeat():
+    w = genome.small_pair(11, length=20000, n_seeds=300)
+    g1, *_ = run_both(w.T, w.Q, w.seeds)
+    g2, *_ = run_both(w.T, w.Q, w.seeds)
+    assert np.array_equal(g1.rec, g2.rec) and g1.cigar == g2.cigar
