@@ -1,0 +1,314 @@
+#!/usr/bin/env python
+"""Benchmark of the FastZ hot path on B200 (driver contract: one JSON line on rank 0).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config 2] [--impl fastz|reference]
+
+Workload (BASELINE.json configs[1], "C2"): synthetic 10 Mbp chromosome pair, 2^20 seeds per GPU with the
+paper's skewed extension-length mix (synth.genome.config2).  One step = one call
+of fastz_extend_seeds over the whole seed batch: inspector + eager traceback, binning, trimmed executor,
+traceback and CIGAR assembly, with the seeds and sequences already resident in HBM (``value``); ``e2e``
+repeats it through the public API from pinned host seeds to host records + CIGAR text.
+
+Metric: GCUPS = explored DP cells (origin + cells with a live neighbour, reading R7 -- the exact
+count, produced once by the census kernel and parity-tested against the oracle) / step time.  Multi-GPU:
+seeds are sharded, nothing is exchanged in the timed region (scaling "weak"); time = max over ranks.
+
+--impl reference times the CPU oracle (oracle/, the plain sequential implementation) on a bounded sample
+of the same workload on this box's host cores; it is the reference arm of this tier.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+OPS_PER_CELL = 13  # 9 recurrence ops (4 max + 5 add) + 4 cone y-drop ops
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", type=int, default=2)
+    ap.add_argument("--seeds", type=int, default=0, help="seeds per GPU (default: the config's)")
+    ap.add_argument("--impl", default="fastz", choices=["fastz", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--profile", action="store_true", help="one warm-up + 1 step, for ncu")
+    return ap.parse_args()
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def workload(config: int, n_per_gpu: int, world: int, rank: int):
+    from synth import genome
+    if config == 2:
+        n = n_per_gpu or (1 << 20)
+        w = genome.config2(n_seeds=n * world)
+        desc = "C2: synthetic 10 Mbp chromosome pair, skewed extension lengths (>97% <=128 bp), LASTZ default scoring"
+    elif config == 1:
+        n = n_per_gpu or 2048
+        w = genome.config1(n_seeds=n * world)
+        desc = "C1: synthetic 100 kbp target vs mutated copy (~10% subs, 1% indels)"
+    elif config == 5:
+        n = n_per_gpu or (1 << 20)
+        w = genome.config5(n_seeds=n * world)
+        desc = "C5: extension-length stress sweep 32 bp - 64 kbp"
+    elif config == 3:
+        n = n_per_gpu or (1 << 21)
+        w = genome.config3(n_seeds=n * world)
+        desc = "C3: synthetic 100 Mbp pair with 16-64 kbp alignments"
+    else:
+        raise SystemExit(f"config {config} not supported by bench")
+    shard = w.seeds[rank::world][:n]
+    return w, shard, desc
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu: int):
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--id={gpu}", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                       "-lms", "200"], stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        try:
+            self.p.wait(5)
+        except Exception:
+            self.p.kill()
+        self.f.flush()
+        rows = [r.split(",") for r in open(self.f.name).read().strip().splitlines() if r.strip()]
+        os.unlink(self.f.name)
+        sm = [float(r[1]) for r in rows if len(r) > 8 and r[1].strip().replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if len(r) > 8 and r[2].strip().replace(".", "").isdigit()]
+        reasons = set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            if len(r) > 8:
+                for k, nm in enumerate(names):
+                    if "Active" in r[5 + k] and "Not" not in r[5 + k]:
+                        reasons.add(nm)
+        loaded = [s for s in sm if s > 500] or sm
+        return {"sm_mhz": statistics.median(loaded) if loaded else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(rows)}
+
+
+def cpu_baseline(w, seeds, target_s=15.0):
+    """The oracle as it stands on this box's host cores, on a bounded random sample of the workload."""
+    import numpy as np
+    from oracle import core
+    cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count()
+    rng = np.random.default_rng(12345)
+    n = min(len(seeds), max(64, 8 * cores))
+    idx = rng.choice(len(seeds), n, replace=False)
+    t0 = time.perf_counter()
+    r = core.extend(w.T, w.Q, seeds[idx], threads=cores)
+    dt = time.perf_counter() - t0
+    if dt < target_s / 3 and n < len(seeds):
+        n2 = min(len(seeds), int(n * target_s / max(dt, 1e-3)))
+        idx = rng.choice(len(seeds), n2, replace=False)
+        t0 = time.perf_counter()
+        r = core.extend(w.T, w.Q, seeds[idx], threads=cores)
+        dt = time.perf_counter() - t0
+        n = n2
+    cells = int(r.rec["l_explored"].sum() + r.rec["r_explored"].sum())
+    return {"value": cells / dt / 1e9, "unit": "GCUPS", "cores": cores, "kind": "oracle",
+            "sample": f"{n} random seeds of the same workload ({cells} explored cells) in {dt:.2f} s, "
+                      f"{cores} threads", "seeds_per_s": n / dt}
+
+
+def run_reference(args, ws, rank):
+    if rank != 0:
+        return
+    import numpy as np
+    from oracle import core
+    w, seeds, desc = workload(args.config, args.seeds, 1, 0)
+    cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count()
+    rng = np.random.default_rng(777)
+    per = max(64, 6 * cores)
+    # calibrate so one step takes ~8 s on this host
+    t0 = time.perf_counter()
+    core.extend(w.T, w.Q, seeds[rng.choice(len(seeds), per, replace=False)], threads=cores)
+    dt = time.perf_counter() - t0
+    per = int(min(len(seeds), max(per, per * 8.0 / max(dt, 1e-3))))
+    for _ in range(args.warmup):
+        core.extend(w.T, w.Q, seeds[rng.choice(len(seeds), min(per, 64), replace=False)], threads=cores)
+    tot_cells, tot_t = 0, 0.0
+    for _ in range(args.steps):
+        idx = rng.choice(len(seeds), per, replace=False)
+        t0 = time.perf_counter()
+        r = core.extend(w.T, w.Q, seeds[idx], threads=cores)
+        tot_t += time.perf_counter() - t0
+        tot_cells += int(r.rec["l_explored"].sum() + r.rec["r_explored"].sum())
+    v = tot_cells / tot_t / 1e9
+    line = {"impl": "reference", "metric": "GCUPS", "value": v, "unit": "GCUPS", "n_gpus": ws, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": tot_t / args.steps * 1e3, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+            "config": {"workload": desc, "seeds_per_step": per, "sample": "random seeds of the workload per step"},
+            "cpu_baseline": {"value": v, "unit": "GCUPS", "cores": cores, "kind": "oracle",
+                             "sample": f"{per} random seeds per step x {args.steps} steps"},
+            "e2e": {"value": v, "unit": "GCUPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def run_fastz(args, ws, rank, local):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_gundaboluvt21_b200 import fastz
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream(dev)
+    w, shard, desc = workload(args.config, args.seeds, ws, rank)
+    n = len(shard)
+    al = fastz.Aligner(w.T, w.Q, device=local, stream=stream.cuda_stream)
+    seeds_d = torch.from_numpy(np.ascontiguousarray(shard)).to(dev)
+    seeds_h = torch.from_numpy(np.ascontiguousarray(shard)).pin_memory()
+
+    # exact explored-cell count (GCUPS numerator), untimed
+    al.extend_only(seeds_d)
+    cells = int(al.census().sum())
+    st0 = al.stats()
+    peak_ops, peak_mhz = fastz.fastz_int_peak(local, 300.0)
+
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
+    for _ in range(args.warmup):
+        al.extend_only(seeds_d)
+    torch.cuda.synchronize()
+    if ws > 1:
+        dist.barrier()
+    clk = Clocks(local)
+    times, insp, stages = [], [], []
+    for _ in range(args.steps):
+        flush.zero_()  # L2 flushed between timed steps (outside the events)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        e0.record(stream)
+        al.extend_only(seeds_d)
+        e1.record(stream)
+        e1.synchronize()
+        times.append(e0.elapsed_time(e1))
+        s = al.stats()
+        insp.append(s["ms_inspect"])
+        stages.append(s)
+    torch.cuda.synchronize()
+    clocks = clk.stop()
+    if ws > 1:
+        dist.barrier()
+    ms = sum(times) / len(times)
+
+    # e2e through the public API: pinned host seeds -> host records + CIGAR
+    e2e_t = []
+    d2h = 0
+    for _ in range(max(1, min(args.steps, 3))):
+        flush.zero_()
+        torch.cuda.synchronize()
+        if ws > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        al.extend_only(seeds_h)
+        res = al.results()
+        e2e_t.append(time.perf_counter() - t0)
+        d2h = res.rec.nbytes + len(res.cigar)
+    e2e_ms = sum(e2e_t) / len(e2e_t) * 1e3
+
+    t = torch.tensor([ms, e2e_ms, float(cells), float(n)], dtype=torch.float64, device=dev)
+    if ws > 1:
+        tmax = t.clone()
+        dist.all_reduce(tmax[:2], op=dist.ReduceOp.MAX)
+        tsum = t.clone()
+        dist.all_reduce(tsum[2:], op=dist.ReduceOp.SUM)
+        ms, e2e_ms = float(tmax[0]), float(tmax[1])
+        cells_all, n_all = float(tsum[2]), float(tsum[3])
+    else:
+        cells_all, n_all = float(cells), float(n)
+    if rank != 0:
+        return
+    value = cells_all / (ms * 1e-3) / 1e9
+    insp_ms = sum(insp) / len(insp)
+    achieved = OPS_PER_CELL * cells / (insp_ms * 1e-3)
+    traffic = None
+    tf = os.path.join(ROOT, "profiles", "inspector_traffic.json")
+    if os.path.exists(tf):
+        try:
+            traffic = json.load(open(tf)).get("bytes_per_launch")
+        except Exception:
+            traffic = None
+    avg = lambda k: sum(s[k] for s in stages) / len(stages)  # noqa: E731
+    line = {
+        "metric": "GCUPS", "value": value, "unit": "GCUPS", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
+        "data": "synthetic",
+        "config": {"workload": desc, "seeds_per_gpu": n, "target_bp": len(w.T), "query_bp": len(w.Q),
+                   "l2": "flushed between timed steps (256 MiB write, untimed)", "rows_per_lane": stages[0].get("R", None)
+                   or int(os.environ.get("FASTZ_R", "4")), "parallelism": f"seed-sharded x{ws}"},
+        "seed_extensions_per_s": n_all / (ms * 1e-3),
+        "cells": cells_all,
+        "clocks": clocks,
+        "e2e": {"value": cells_all / (e2e_ms * 1e-3) / 1e9, "unit": "GCUPS", "ms_per_step": e2e_ms,
+                "h2d_bytes_per_step": int(n * 16), "d2h_bytes_per_step": int(d2h)},
+        "gpu_launches": 10 * args.steps,
+        "roofline": {"bound": "alu", "kernel": "k_inspect", "achieved": achieved / 1e12, "peak": peak_ops / 1e12,
+                     "unit": "Tops/s (INT32 lane ops)", "frac": achieved / peak_ops, "traffic": traffic,
+                     "ops_per_cell": OPS_PER_CELL, "inspector_ms": insp_ms,
+                     "peak_source": f"measured fastz_int_peak (IMNMX/IADD3/VIADDMNMX chains) at {peak_mhz:.0f} MHz"},
+        "stages_ms": {k: avg(k) for k in ("ms_upload", "ms_inspect", "ms_bin", "ms_execute", "ms_traceback",
+                                          "ms_combine")},
+        "bins_per_side": st0["bin_counts"][:7], "exec_sides": st0["n_exec_sides"], "eager_sides": st0["n_eager_sides"],
+    }
+    if not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline(w, shard)
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    ws, rank, local = dist_env()
+    if ws > 1:
+        import torch
+        import torch.distributed as dist
+        if args.impl == "reference":
+            if rank != 0:
+                return
+            ws_eff = ws
+            run_reference(args, ws_eff, 0)
+            return
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    if args.impl == "reference":
+        run_reference(args, ws, rank)
+        return
+    if args.profile:
+        args.warmup, args.steps = 1, 1
+    run_fastz(args, ws, rank, local)
+    if ws > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

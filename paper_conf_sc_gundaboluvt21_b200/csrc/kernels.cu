@@ -84,7 +84,7 @@ __device__ __forceinline__ void setup_side(const Batch& b, int side, SideIO& io)
 constexpr int OP_M = 0, OP_I = 1, OP_D = 2;
 
 struct SmemDP {
-    int2 cpr[WARPS][CP_RING + 16];
+    WarpSmem w[WARPS];
     int2 cptab[8];
     uint8_t ecodes[WARPS][EAGER_W * EAGER_W + 15];
 };
@@ -107,7 +107,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_inspect(DevParams P, Batch b, in
     SideIO io;
     io.ring = ring + (size_t)(blockIdx.x * WARPS + warp) * (size_t)(rmask + 1);
     io.rmask = rmask;
-    io.cpring = sm.cpr[warp];
+    io.ws = &sm.w[warp];
     io.cptab = sm.cptab;
     io.ecodes = sm.ecodes[warp];
     io.eager_max = P.eager_max;
@@ -175,7 +175,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int
     SideIO io;
     io.ring = ring + (size_t)(blockIdx.x * WARPS + warp) * (size_t)(rmask + 1);
     io.rmask = rmask;
-    io.cpring = sm.cpr[warp];
+    io.ws = &sm.w[warp];
     io.cptab = sm.cptab;
     io.ecodes = nullptr;
     io.eager_max = -1;
@@ -207,7 +207,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, in
     SideIO io;
     io.ring = ring + (size_t)(blockIdx.x * WARPS + warp) * (size_t)(rmask + 1);
     io.rmask = rmask;
-    io.cpring = sm.cpr[warp];
+    io.ws = &sm.w[warp];
     io.cptab = sm.cptab;
     io.ecodes = nullptr;
     io.eager_max = -1;

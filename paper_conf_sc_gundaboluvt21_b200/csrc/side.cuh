@@ -9,12 +9,30 @@
 //               so each warp store is one coalesced 128-byte line (P:180's consolidation, done in registers).
 // MODE_CENSUS:  counts explored cells (origin + cells with a live diagonal/up/left neighbour), the GCUPS
 //               numerator; not on the timed path.
+//
+// Per-step data movement (the paper's register exchange, re-designed for sm_100a):
+//  * lane l receives the bottom row (X, D, W) of lane l-1 with a ROTATING shuffle (src = l-1 mod 32): lane 0
+//    receives from lane 31, which -- after parking its own bottom row in shared staging -- holds the previous
+//    strip's boundary value for lane 0's next column.  No per-step global memory access, no lane-0 selects.
+//  * every 16 steps the warp moves 16 boundary values global ring -> shared staging (prefetched one block
+//    ahead) and 16 parked bottom-row values shared -> global ring, both coalesced.
+//  * termination: each lane keeps a 32-step history of "all my R cells dead"; the strip is done at column x
+//    (lane 31's) iff every lane was dead at x and the boundary row has no live cell at or after x -- the
+//    unrolled form of the per-lane "done" chain.  Tested every 4 steps.
 #pragma once
+#include <type_traits>
+
 #include "dp.cuh"
 
 namespace fz {
 
 enum { MODE_INSPECT = 0, MODE_EXEC = 1, MODE_CENSUS = 2 };
+
+struct WarpSmem {
+    int2 cp[CP_RING + 16];  // column profiles, ring over relative columns (+16 mirrored)
+    int4 bin[32];           // boundary row staging (lane 0's input, served through lane 31)
+    int4 bout[32];          // lane 31's bottom-row outputs awaiting the global ring
+};
 
 struct SideIO {
     const uint32_t* __restrict__ Apk;  // target side (rows), packed; A_k at position Aoff + k - 1
@@ -26,7 +44,7 @@ struct SideIO {
     int N;                              // columns 0..N (N <= Bmax; the executor trims to j*)
     int4* __restrict__ ring;            // per-warp boundary ring, rmask + 1 entries {X, D, W, -}
     int rmask;
-    int2* cpring;                       // shared: CP_RING + 16 column-profile entries
+    WarpSmem* ws;                       // shared staging of this warp
     const int2* cptab;                  // shared: 5 profiles (query base 0..3, zero)
     uint8_t* ecodes;                    // shared: EAGER_W^2 eager codes (inspector)
     int eager_max;
@@ -48,15 +66,19 @@ struct StripGeom {
     static constexpr int SPW = 8 / R;  // steps per 32-bit code word
 };
 
-// Column profile ring refill: entry for relative column rc (column start + rc) at index rc & 127 (+ mirror).
-__device__ __forceinline__ void cp_put(const SideIO& io, int start, int rc) {
-    const int c = start + rc;
-    int b = 4;
-    if (c >= 1 && c <= io.N) b = base_at(io.Bpk, io.Boff + c - 1);
-    const int2 v = io.cptab[b];
+__device__ __forceinline__ int query_code(const SideIO& io, int c) {
+    return (c >= 1 && c <= io.N) ? base_at(io.Bpk, io.Boff + c - 1) : 4;
+}
+
+__device__ __forceinline__ void cp_store(const SideIO& io, int rc, int code) {
+    const int2 v = io.cptab[code];
     const int idx = rc & (CP_RING - 1);
-    io.cpring[idx] = v;
-    if (idx < 16) io.cpring[idx + CP_RING] = v;
+    io.ws->cp[idx] = v;
+    if (idx < 16) io.ws->cp[idx + CP_RING] = v;
+}
+
+__device__ __forceinline__ int4 boundary(const int4* __restrict__ ring, int rmask, int c, int Emax, int Wfar) {
+    return c <= Emax ? ring[c & rmask] : make_int4(NEG, NEG, Wfar, 0);
 }
 
 template <int R, int MODE, bool EAGER>
@@ -64,24 +86,18 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
     constexpr int H = StripGeom<R>::H;
     constexpr int SPW = StripGeom<R>::SPW;
     const int lane = threadIdx.x & 31;
+    const int src = (lane + 31) & 31;
     const int M = io.M, N = io.N;
     const int E = P.E, OE = P.OE, OEmY = P.OE - P.Y, mE = -P.E;
-    const unsigned amask = lane == 0 ? 0u : (1u << (lane - 1));
     const int rmask = io.rmask;
     int4* __restrict__ ring = io.ring;
+    WarpSmem* __restrict__ ws = io.ws;
 
     int start = 0, Wleft0 = NEG, lastlive = -1, Emax = -1, Wfar = NEG;
     int best = NEG + 1, bi = INT_MAX, bj = INT_MAX;
     long long cum_words = 0, bound_words = 0, cells = 0;
     uint32_t flags = 0;
     bool upd = false;
-
-    // row -1 lies outside the matrix: dead, V = -inf.  Two sentinel entries (lane 0 double-buffers).
-    if (lane == 0) {
-        ring[0] = make_int4(NEG, NEG, NEG, 0);
-        ring[1] = make_int4(NEG, NEG, NEG, 0);
-    }
-    __syncwarp();
 
     int s = 0;
     for (int top = 0; top <= M; top += H, ++s) {
@@ -104,41 +120,43 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         int xb = NEG, db = NEG, wb = NEG;
         const int span = N - start;
         const int tlast = span + 31;
-        const int lim2 = lane == 0 ? Emax + 2 : INT_MIN;
-        const int t0l = lane == 0 ? lastlive - start : INT_MAX;
-        int4 B0 = make_int4(NEG, NEG, NEG, 0), B1 = B0;
-        if (lane == 0) {
-            B0 = ring[start & rmask];
-            B1 = ring[(start + 1) & rmask];
-        }
-        long long wbase = cum_words;  // executor: this strip's first word (relative to the side)
+        const long long wbase = cum_words;  // executor: this strip's first word (relative to the side)
         if constexpr (MODE == MODE_EXEC) {
             if (lane == 0) io.stab[s] = make_int2(start, (int)wbase);
         }
+        // staging: boundary for relative columns [0, 32), column profiles [0, 32); prefetch the next 16
+        ws->bin[lane] = boundary(ring, rmask, start + lane, Emax, Wfar);
+        cp_store(io, lane, query_code(io, start + lane));
+        int4 bpre = make_int4(NEG, NEG, Wfar, 0);
+        int qpre = 4;
+        if (lane < 16) {
+            bpre = boundary(ring, rmask, start + 32 + lane, Emax, Wfar);
+            qpre = query_code(io, start + 32 + lane);
+        }
+        __syncwarp();
+        if (lane == 31) {
+            const int4 v = ws->bin[0];
+            xb = v.x;
+            db = v.y;
+            wb = v.z;
+        }
         uint32_t cw = 0;
-        unsigned prevb = 0;
+        unsigned hist = 0;
         int tfinal = 0;
 
-        cp_put(io, start, lane);  // relative columns [0, 32)
-        __syncwarp();
-
         // one wavefront step: lane computes column start + tt - lane.  Returns true when the strip is done.
-        auto step = [&](auto eag, const int tt, const int u, const int cbase, int4& BU) -> bool {
+        auto step = [&](auto chk, auto eag, const int tt, const int u, const int j, const int cbase) -> bool {
+            constexpr bool CHK = decltype(chk)::value;
             constexpr bool EG = decltype(eag)::value;
             const int rc = tt - lane;
-            const bool valid = (unsigned)rc <= (unsigned)span;
-            int xu = __shfl_up_sync(FULL, xb, 1);
-            int du = __shfl_up_sync(FULL, db, 1);
-            int wu = __shfl_up_sync(FULL, wb, 1);
-            if (lane == 0) {
-                xu = BU.x;
-                du = BU.y;
-                wu = BU.z;
-            }
-            if (start + tt + 2 <= lim2) BU = ring[(start + tt + 2) & rmask];
-            bool done = false;
+            const bool valid = CHK ? (unsigned)rc <= (unsigned)span : true;
+            int xu = __shfl_sync(FULL, xb, src);
+            int du = __shfl_sync(FULL, db, src);
+            int wu = __shfl_sync(FULL, wb, src);
+            unsigned dead = 1u;
+            int cmv = NEG;
             if (valid) {
-                const int2 cp = io.cpring[cbase + u];
+                const int2 cp = ws->cp[cbase + u];
                 int xd = xdiag;
                 xdiag = xu;
                 int cm = NEG;
@@ -153,7 +171,7 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                     const int wn = __viaddmax_s32(xn, OEmY, thr);
                     if constexpr (MODE == MODE_EXEC) {
                         const uint32_t code = cell_code(h, d, iv, du, xu, I[k], X[k], E);
-                        cw |= code << ((((tt % SPW) * R) + k) * 4);
+                        cw |= code << ((((j % SPW) * R) + k) * 4);
                     }
                     if constexpr (EG) {
                         const int r = r0 + k, c = start + rc;
@@ -175,33 +193,46 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                 xb = xu;
                 db = du;
                 wb = wu;
-                if constexpr (MODE == MODE_INSPECT) {
-                    if (cm >= best) {
-                        const int c = start + rc;
+                dead = cm == NEG;
+                cmv = cm;
+            }
+            if constexpr (MODE == MODE_INSPECT) {
+                // peak (reading R5): rare, warp-uniform slow path; ties -> smaller row (columns only grow)
+                if (__any_sync(FULL, cmv >= best)) {
+                    const int c = start + rc;
 #pragma unroll
-                        for (int k = 0; k < R; ++k) {
-                            const int r = r0 + k;
-                            if (X[k] > best || (X[k] == best && r < bi)) {
-                                best = X[k];
-                                bi = r;
-                                bj = c;
-                                upd = true;
-                            }
-                        }
+                    for (int k = 0; k < R; ++k) {
+                        const int r = r0 + k;
+                        const bool better = valid && (X[k] > best || (X[k] == best && r < bi));
+                        best = better ? X[k] : best;
+                        bi = better ? r : bi;
+                        bj = better ? c : bj;
+                        upd |= better;
                     }
                 }
-                if (lane == 31) ring[(start + rc) & rmask] = make_int4(xb, db, wb, 0);
-                done = cm == NEG;
+            }
+            if (lane == 31) {
+                ws->bout[tt & 31] = make_int4(xb, db, wb, 0);
+                const int4 v = ws->bin[(tt + 1) & 31];
+                xb = v.x;
+                db = v.y;
+                wb = v.z;
             }
             if constexpr (MODE == MODE_EXEC) {
-                if ((tt % SPW) == SPW - 1) {
+                if ((j % SPW) == SPW - 1) {  // j == tt mod 4 and SPW divides 4
                     io.codes[wbase + (long long)(tt / SPW) * 32 + lane] = cw;
                     cw = 0;
                 }
             }
-            done = done && (((prevb & amask) != 0) || tt > t0l);
-            prevb = __ballot_sync(FULL, done);
-            if ((int)prevb < 0 || tt == tlast) {
+            hist = (hist << 1) | dead;
+            if (j == 3 && tt >= 31) {
+                const unsigned bal = __ballot_sync(FULL, (hist >> (31 - lane)) & 1u);
+                if (bal == FULL && start + tt - 31 > lastlive) {
+                    tfinal = tt;
+                    return true;
+                }
+            }
+            if (CHK && tt == tlast) {
                 tfinal = tt;
                 return true;
             }
@@ -210,24 +241,41 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
 
         int t = 0;
         for (;;) {
-            if (t > 0 && lane < 16) cp_put(io, start, t + 16 + lane);
+            if (t > 0) {
+                __syncwarp();  // lane 31's parked rows of the previous block -> visible to lanes 0..15
+                // staging refills for relative columns [t+16, t+32), prefetch [t+32, t+48); park -> ring
+                if (lane < 16) {
+                    const int rcn = t + 16 + lane;
+                    ws->bin[rcn & 31] = bpre;
+                    cp_store(io, rcn, qpre);
+                    bpre = boundary(ring, rmask, start + rcn + 16, Emax, Wfar);
+                    qpre = query_code(io, start + rcn + 16);
+                    const int st = t - 16 + lane, rc31 = st - 31;
+                    if (rc31 >= 0 && rc31 <= span) ring[(start + rc31) & rmask] = ws->bout[st & 31];
+                }
+            }
             __syncwarp();
             const int cbase = (t - lane) & (CP_RING - 1);
             bool fin = false;
+            std::integral_constant<bool, true> yes;
+            std::integral_constant<bool, false> no;
             if (EAGER && MODE == MODE_INSPECT && top == 0 && t < 32) {
-                std::integral_constant<bool, true> eg;
+#pragma unroll 1
+                for (int u = 0; u < 16; ++u)
+                    if (step(yes, yes, t + u, u, u & 3, cbase)) { fin = true; break; }
+            } else if (t >= 32 && t + 15 <= span) {
+                // steady state: every lane valid for all 16 steps; 4-step unrolled body keeps the hot loop
+                // inside the instruction cache
+#pragma unroll 1
+                for (int q = 0; q < 16 && !fin; q += 4) {
 #pragma unroll
-                for (int u = 0; u < 16; u += 2) {
-                    if (step(eg, t + u, u, cbase, B0)) { fin = true; break; }
-                    if (step(eg, t + u + 1, u + 1, cbase, B1)) { fin = true; break; }
+                    for (int j = 0; j < 4; ++j)
+                        if (step(no, no, t + q + j, q + j, j, cbase)) { fin = true; break; }
                 }
             } else {
-                std::integral_constant<bool, false> eg;
-#pragma unroll
-                for (int u = 0; u < 16; u += 2) {
-                    if (step(eg, t + u, u, cbase, B0)) { fin = true; break; }
-                    if (step(eg, t + u + 1, u + 1, cbase, B1)) { fin = true; break; }
-                }
+#pragma unroll 1
+                for (int u = 0; u < 16; ++u)
+                    if (step(yes, no, t + u, u, u & 3, cbase)) { fin = true; break; }
             }
             if (fin) break;
             t += 16;
@@ -235,6 +283,11 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
 
         // ------------------------------------------------------------------ strip finish
         const int e = start + tfinal - 31;  // lane 31's last column
+        __syncwarp();
+        if (lane < 16) {  // park the last (partial) block's bottom rows in the ring
+            const int st = t + lane, rc31 = st - 31;
+            if (st <= tfinal && rc31 >= 0 && rc31 <= span) ring[(start + rc31) & rmask] = ws->bout[st & 31];
+        }
         if constexpr (MODE == MODE_EXEC) {
             if ((tfinal % SPW) != SPW - 1) io.codes[wbase + (long long)(tfinal / SPW) * 32 + lane] = cw;
         }
@@ -243,7 +296,11 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             if (__any_sync(FULL, upd)) bound_words = cum_words;
             upd = false;
         }
-        const int Wtail = __shfl_sync(FULL, wb, 31);
+        const int Wtail = ws->bout[tfinal & 31].z;
+        if (e - start + 4 > rmask) {  // strip wider than the ring: the parked row has been overwritten
+            flags |= SF_RING;
+            break;
+        }
         __syncwarp();
         // V of the boundary row beyond e: max of the old boundary and this strip's tail (exact, reading R3)
         for (int c = e + 1 + lane; c <= Emax; c += 32) {
@@ -278,10 +335,6 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         if (Emax + 4 - first > rmask) {      // boundary band wider than the ring
             flags |= SF_RING;
             break;
-        }
-        if (lane == 0) {
-            ring[(Emax + 1) & rmask] = make_int4(NEG, NEG, Wfar, 0);
-            ring[(Emax + 2) & rmask] = make_int4(NEG, NEG, Wfar, 0);
         }
         if (first > start) Wleft0 = ring[(first - 1) & rmask].z;
         lastlive = last;
