@@ -36,11 +36,41 @@ constexpr int EAGER_W = 17;       // eager code window: rows/cols 0..16 (P:168, 
 constexpr uint32_t SF_EAGER = 1u, SF_OVERFLOW = 2u, SF_RING = 4u, SF_EXEC_MISMATCH = 8u;
 
 struct DevParams {
-    int cp[10];        // column profile per query base b (0..3) and the zero profile (b = 4):
-                       //   cp[2b] = (sub(A,b) & 0xffff) | sub(C,b) << 16, cp[2b+1] = (sub(G,b) & 0xffff) | sub(T,b) << 16
+    int cp[10];        // column profile per query base b (0..3) and the origin profile (b = 4):
+                       //   cp[2b] = (v(A,b) & 0xffff) | v(C,b) << 16, cp[2b+1] = (v(G,b) & 0xffff) | v(T,b) << 16
+                       //   with v = sub + O + E when every such value fits int16 (fold_oe = 1), else v = sub
     int O, E, Y, OE;   // gap open, extend, y-drop, O+E
     int K, eager_max;
+    int fold_oe;       // O+E folded into the profile (H = X_diag + v) -- see cp above
+    int one, zero;     // runtime 1 and 0: keep adds/selects as IMAD on the FMA pipe (ALU pipe is the limiter)
 };
+
+// d = a * one + c on the FMA pipe (one == 1 at run time; ptxas cannot fold it into an ALU IADD3)
+__device__ __forceinline__ int fma_add(int a, int one, int c) {
+    int d;
+    asm("mad.lo.s32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(one), "r"(c));
+    return d;
+}
+
+// y-drop kill (reading R3) with the select on the FMA pipe: x = (s >= thr) ? s - OE : NEG
+__device__ __forceinline__ int kill_fma(int s, int thr, int mOE, int one, int zero) {
+    int x = fma_add(s, one, mOE);
+    // x * zero + NEG depends on x, so ptxas cannot hoist it into a SEL on the ALU pipe
+    asm("{ .reg .pred p; setp.lt.s32 p, %1, %2; @p mad.lo.s32 %0, %0, %3, %4; }"
+        : "+r"(x) : "r"(s), "r"(thr), "r"(zero), "n"(NEG));
+    return x;
+}
+
+// predicated shared-memory store / load (keeps per-lane staging as predicated instructions, not a branch)
+__device__ __forceinline__ void st_shared_if(bool p, unsigned addr, int v) {
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %0, 0; @q st.shared.b32 [%1], %2; }" ::"r"((unsigned)p), "r"(addr),
+                 "r"(v)
+                 : "memory");
+}
+__device__ __forceinline__ void ld_shared_if(bool p, unsigned addr, int& v) {
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %1, 0; @q ld.shared.b32 %0, [%2]; }" : "+r"(v) : "r"((unsigned)p), "r"(addr)
+                 : "memory");
+}
 
 __device__ __forceinline__ int prmt(int a, int b, int s) {
     int d;

@@ -98,7 +98,7 @@ __device__ __forceinline__ void smem_init(SmemDP& sm, const DevParams& P) {
 // Persistent: each warp pops one-sided extensions from an atomic queue (load balance replaces the paper's
 // 32 CUDA streams).  Score-only DP + eager 17x17 corner codes; when the peak lies inside the
 // eager window the warp's lane 0 walks the codes at once and the side skips the executor.
-template <int R>
+template <int R, bool FOLD>
 __global__ void __launch_bounds__(WARPS * 32) k_inspect(DevParams P, Batch b, int4* ring, int rmask,
                                                          SideArrays sa, int* counter) {
     __shared__ SmemDP sm;
@@ -121,7 +121,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_inspect(DevParams P, Batch b, in
         if (side >= nsides) break;
         setup_side(b, side, io);
         SideOut o;
-        run_side<R, MODE_INSPECT, true>(P, io, o);
+        run_side<R, MODE_INSPECT, true, FOLD>(P, io, o);
         __syncwarp();  // eager corner codes (shared memory) written by lanes 0..4 -> read by lane 0
         if (lane == 0) {
             uint32_t flags = o.flags;
@@ -166,7 +166,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_inspect(DevParams P, Batch b, in
     }
 }
 
-template <int R>
+template <int R, bool FOLD>
 __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int4* ring, int rmask,
                                                         long long* cells, int* counter) {
     __shared__ SmemDP sm;
@@ -189,7 +189,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int
         if (side >= nsides) break;
         setup_side(b, side, io);
         SideOut o;
-        run_side<R, MODE_CENSUS, false>(P, io, o);
+        run_side<R, MODE_CENSUS, false, FOLD>(P, io, o);
         if (lane == 0) cells[side] = (o.flags & SF_RING) ? -1 : o.cells;
         __syncwarp();
     }
@@ -198,7 +198,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int
 // ------------------------------------------------------------------------------------------------- executor
 // Trimmed executor: the DP over [0,i*]x[0,j*] only, writing traceback codes.  Persistent warps
 // pop non-eager sides in bin order, largest bins first (length binning P:209-211 used as an LPT schedule).
-template <int R>
+template <int R, bool FOLD>
 __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, int4* ring, int rmask,
                                                          SideArrays sa, ExecPlan pl, int nexec, Outputs out) {
     __shared__ SmemDP sm;
@@ -223,7 +223,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, in
         io.codes = out.codes + pl.woff[side];
         io.stab = out.stab + pl.soff[side];
         SideOut o;
-        run_side<R, MODE_EXEC, false>(P, io, o);
+        run_side<R, MODE_EXEC, false, FOLD>(P, io, o);
         if (lane == 0 && (o.flags & SF_RING)) atomicOr(&sa.flags[side], SF_RING);
         __syncwarp();
     }
@@ -347,7 +347,6 @@ cudaError_t launch_bin(int R, const SideArrays& sa, int nsides, const ExecPlan& 
         const int g = (nsides + 255) / 256;
         switch (R) {
             case 2: k_bin_count<2><<<g, 256, 0, st>>>(sa, nsides, pl, words, strips, runs); break;
-            case 8: k_bin_count<8><<<g, 256, 0, st>>>(sa, nsides, pl, words, strips, runs); break;
             default: k_bin_count<4><<<g, 256, 0, st>>>(sa, nsides, pl, words, strips, runs); break;
         }
         cudaError_t e;
@@ -493,7 +492,7 @@ int pick_R() {
     if (!r) {
         const char* e = getenv("FASTZ_R");
         r = e ? atoi(e) : 4;
-        if (r != 2 && r != 4 && r != 8) r = 4;
+        if (r != 2 && r != 4) r = 4;
     }
     return r;
 }
@@ -501,48 +500,41 @@ int pick_R() {
 template <int R>
 static int bps_of() {
     int n = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_inspect<R>, WARPS * 32, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_inspect<R, true>, WARPS * 32, 0);
     return n > 0 ? n : 1;
 }
 
-int inspector_blocks_per_sm(int R) {
-    switch (R) {
-        case 2: return bps_of<2>();
-        case 8: return bps_of<8>();
-        default: return bps_of<4>();
-    }
-}
+int inspector_blocks_per_sm(int R) { return R == 2 ? bps_of<2>() : bps_of<4>(); }
+
+#define FZ_DISPATCH(KERNEL, GRID, ...)                                                   \
+    do {                                                                                 \
+        if (R == 2) {                                                                    \
+            if (P.fold_oe) KERNEL<2, true><<<GRID, WARPS * 32, 0, st>>>(__VA_ARGS__);    \
+            else KERNEL<2, false><<<GRID, WARPS * 32, 0, st>>>(__VA_ARGS__);             \
+        } else {                                                                         \
+            if (P.fold_oe) KERNEL<4, true><<<GRID, WARPS * 32, 0, st>>>(__VA_ARGS__);    \
+            else KERNEL<4, false><<<GRID, WARPS * 32, 0, st>>>(__VA_ARGS__);             \
+        }                                                                                \
+    } while (0)
 
 cudaError_t launch_inspect(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
                            const SideArrays& sa, int* counter, cudaStream_t st) {
     if (b.nseeds == 0) return cudaSuccess;
-    switch (R) {
-        case 2: k_inspect<2><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, counter); break;
-        case 8: k_inspect<8><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, counter); break;
-        default: k_inspect<4><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, counter); break;
-    }
+    FZ_DISPATCH(k_inspect, grid, P, b, ring, rmask, sa, counter);
     return cudaGetLastError();
 }
 
 cudaError_t launch_census(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
                           long long* cells, int* counter, cudaStream_t st) {
     if (b.nseeds == 0) return cudaSuccess;
-    switch (R) {
-        case 2: k_census<2><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, cells, counter); break;
-        case 8: k_census<8><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, cells, counter); break;
-        default: k_census<4><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, cells, counter); break;
-    }
+    FZ_DISPATCH(k_census, grid, P, b, ring, rmask, cells, counter);
     return cudaGetLastError();
 }
 
 cudaError_t launch_execute(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
                            const SideArrays& sa, const ExecPlan& pl, int nexec, const Outputs& o, cudaStream_t st) {
     if (nexec == 0) return cudaSuccess;
-    switch (R) {
-        case 2: k_execute<2><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, pl, nexec, o); break;
-        case 8: k_execute<8><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, pl, nexec, o); break;
-        default: k_execute<4><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, pl, nexec, o); break;
-    }
+    FZ_DISPATCH(k_execute, grid, P, b, ring, rmask, sa, pl, nexec, o);
     return cudaGetLastError();
 }
 
@@ -552,7 +544,6 @@ cudaError_t launch_traceback(int R, const SideArrays& sa, const ExecPlan& pl, in
     const int g = (nexec + 127) / 128;
     switch (R) {
         case 2: k_traceback<2><<<g, 128, 0, st>>>(sa, pl, nexec, o); break;
-        case 8: k_traceback<8><<<g, 128, 0, st>>>(sa, pl, nexec, o); break;
         default: k_traceback<4><<<g, 128, 0, st>>>(sa, pl, nexec, o); break;
     }
     return cudaGetLastError();

@@ -16,9 +16,10 @@
 //    strip's boundary value for lane 0's next column.  No per-step global memory access, no lane-0 selects.
 //  * every 16 steps the warp moves 16 boundary values global ring -> shared staging (prefetched one block
 //    ahead) and 16 parked bottom-row values shared -> global ring, both coalesced.
-//  * termination: each lane keeps a 32-step history of "all my R cells dead"; the strip is done at column x
-//    (lane 31's) iff every lane was dead at x and the boundary row has no live cell at or after x -- the
-//    unrolled form of the per-lane "done" chain.  Tested every 4 steps.
+//  * termination: each lane keeps the last step at which one of its R cells was live; the strip is done at
+//    column x (lane 31's) iff no lane has had a live cell since it processed x and the boundary row has no
+//    live cell at or after x -- the unrolled form of the per-lane "done" chain (lane l is done at x iff its
+//    cells are dead at x and lane l-1 is done at x).  Tested every 4 steps.
 #pragma once
 #include <type_traits>
 
@@ -30,8 +31,8 @@ enum { MODE_INSPECT = 0, MODE_EXEC = 1, MODE_CENSUS = 2 };
 
 struct WarpSmem {
     int2 cp[CP_RING + 16];  // column profiles, ring over relative columns (+16 mirrored)
-    int4 bin[32];           // boundary row staging (lane 0's input, served through lane 31)
-    int4 bout[32];          // lane 31's bottom-row outputs awaiting the global ring
+    int bin[3][32];         // boundary row staging (X, D, W; lane 0's input, served through lane 31)
+    int bout[3][32];        // lane 31's bottom-row outputs (X, D, W) awaiting the global ring
 };
 
 struct SideIO {
@@ -81,17 +82,21 @@ __device__ __forceinline__ int4 boundary(const int4* __restrict__ ring, int rmas
     return c <= Emax ? ring[c & rmask] : make_int4(NEG, NEG, Wfar, 0);
 }
 
-template <int R, int MODE, bool EAGER>
+template <int R, int MODE, bool EAGER, bool FOLD>
 __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, SideOut& out) {
     constexpr int H = StripGeom<R>::H;
     constexpr int SPW = StripGeom<R>::SPW;
     const int lane = threadIdx.x & 31;
     const int src = (lane + 31) & 31;
     const int M = io.M, N = io.N;
-    const int E = P.E, OE = P.OE, OEmY = P.OE - P.Y, mE = -P.E;
+    const int E = P.E, OE = P.OE, OEmY = P.OE - P.Y, mE = -P.E, mOE = -P.OE;
+    const int one = P.one, zero = P.zero;
     const int rmask = io.rmask;
     int4* __restrict__ ring = io.ring;
     WarpSmem* __restrict__ ws = io.ws;
+    const bool is31 = lane == 31;
+    const unsigned sb_in = (unsigned)__cvta_generic_to_shared(&ws->bin[0][0]);
+    const unsigned sb_out = (unsigned)__cvta_generic_to_shared(&ws->bout[0][0]);
 
     int start = 0, Wleft0 = NEG, lastlive = -1, Emax = -1, Wfar = NEG;
     int best = NEG + 1, bi = INT_MAX, bj = INT_MAX;
@@ -125,7 +130,12 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             if (lane == 0) io.stab[s] = make_int2(start, (int)wbase);
         }
         // staging: boundary for relative columns [0, 32), column profiles [0, 32); prefetch the next 16
-        ws->bin[lane] = boundary(ring, rmask, start + lane, Emax, Wfar);
+        {
+            const int4 v = boundary(ring, rmask, start + lane, Emax, Wfar);
+            ws->bin[0][lane] = v.x;
+            ws->bin[1][lane] = v.y;
+            ws->bin[2][lane] = v.z;
+        }
         cp_store(io, lane, query_code(io, start + lane));
         int4 bpre = make_int4(NEG, NEG, Wfar, 0);
         int qpre = 4;
@@ -135,13 +145,12 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         }
         __syncwarp();
         if (lane == 31) {
-            const int4 v = ws->bin[0];
-            xb = v.x;
-            db = v.y;
-            wb = v.z;
+            xb = ws->bin[0][0];
+            db = ws->bin[1][0];
+            wb = ws->bin[2][0];
         }
         uint32_t cw = 0;
-        unsigned hist = 0;
+        int lastlive_t = -1;   // last step at which this lane had a live cell (termination, see header)
         int tfinal = 0;
 
         // one wavefront step: lane computes column start + tt - lane.  Returns true when the strip is done.
@@ -153,7 +162,6 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             int xu = __shfl_sync(FULL, xb, src);
             int du = __shfl_sync(FULL, db, src);
             int wu = __shfl_sync(FULL, wb, src);
-            unsigned dead = 1u;
             int cmv = NEG;
             if (valid) {
                 const int2 cp = ws->cp[cbase + u];
@@ -162,12 +170,13 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                 int cm = NEG;
 #pragma unroll
                 for (int k = 0; k < R; ++k) {
-                    const int h = xd + prmt(cp.x, cp.y, sel[k]) + OE;
+                    const int h = FOLD ? fma_add(prmt(cp.x, cp.y, sel[k]), one, xd)
+                                       : xd + prmt(cp.x, cp.y, sel[k]) + OE;
                     const int d = __viaddmax_s32(du, mE, xu);
                     const int iv = __viaddmax_s32(I[k], mE, X[k]);
                     const int sr = __vimax3_s32(h, d, iv);
                     const int thr = imax(wu, W[k]);
-                    const int xn = (sr >= thr) ? sr - OE : NEG;
+                    const int xn = kill_fma(sr, thr, mOE, one, zero);
                     const int wn = __viaddmax_s32(xn, OEmY, thr);
                     if constexpr (MODE == MODE_EXEC) {
                         const uint32_t code = cell_code(h, d, iv, du, xu, I[k], X[k], E);
@@ -188,12 +197,13 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                     xu = xn;
                     du = d;
                     wu = wn;
-                    cm = imax(cm, xn);
+                    cm = k == 0 ? xn : imax(cm, xn);
                 }
                 xb = xu;
                 db = du;
                 wb = wu;
-                dead = cm == NEG;
+                // live -> tt, dead (cm == NEG) -> -1: one VIADDMNMX (min) + one max
+                lastlive_t = imax(lastlive_t, __viaddmin_s32(cm, -NEG - 1, tt));
                 cmv = cm;
             }
             if constexpr (MODE == MODE_INSPECT) {
@@ -211,12 +221,14 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                     }
                 }
             }
-            if (lane == 31) {
-                ws->bout[tt & 31] = make_int4(xb, db, wb, 0);
-                const int4 v = ws->bin[(tt + 1) & 31];
-                xb = v.x;
-                db = v.y;
-                wb = v.z;
+            {
+                const unsigned o = (unsigned)(tt & 31) * 4u, n = (unsigned)((tt + 1) & 31) * 4u;
+                st_shared_if(is31, sb_out + o, xb);
+                st_shared_if(is31, sb_out + 128u + o, db);
+                st_shared_if(is31, sb_out + 256u + o, wb);
+                ld_shared_if(is31, sb_in + n, xb);
+                ld_shared_if(is31, sb_in + 128u + n, db);
+                ld_shared_if(is31, sb_in + 256u + n, wb);
             }
             if constexpr (MODE == MODE_EXEC) {
                 if ((j % SPW) == SPW - 1) {  // j == tt mod 4 and SPW divides 4
@@ -224,9 +236,10 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                     cw = 0;
                 }
             }
-            hist = (hist << 1) | dead;
             if (j == 3 && tt >= 31) {
-                const unsigned bal = __ballot_sync(FULL, (hist >> (31 - lane)) & 1u);
+                // done at lane 31's column x = start + tt - 31 iff every lane has been dead since it processed
+                // x (step tt - 31 + lane) and the boundary row has no live cell at or after x
+                const unsigned bal = __ballot_sync(FULL, lastlive_t < tt - 31 + lane);
                 if (bal == FULL && start + tt - 31 > lastlive) {
                     tfinal = tt;
                     return true;
@@ -246,12 +259,16 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                 // staging refills for relative columns [t+16, t+32), prefetch [t+32, t+48); park -> ring
                 if (lane < 16) {
                     const int rcn = t + 16 + lane;
-                    ws->bin[rcn & 31] = bpre;
+                    ws->bin[0][rcn & 31] = bpre.x;
+                    ws->bin[1][rcn & 31] = bpre.y;
+                    ws->bin[2][rcn & 31] = bpre.z;
                     cp_store(io, rcn, qpre);
                     bpre = boundary(ring, rmask, start + rcn + 16, Emax, Wfar);
                     qpre = query_code(io, start + rcn + 16);
                     const int st = t - 16 + lane, rc31 = st - 31;
-                    if (rc31 >= 0 && rc31 <= span) ring[(start + rc31) & rmask] = ws->bout[st & 31];
+                    if (rc31 >= 0 && rc31 <= span)
+                        ring[(start + rc31) & rmask] =
+                            make_int4(ws->bout[0][st & 31], ws->bout[1][st & 31], ws->bout[2][st & 31], 0);
                 }
             }
             __syncwarp();
@@ -286,7 +303,9 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         __syncwarp();
         if (lane < 16) {  // park the last (partial) block's bottom rows in the ring
             const int st = t + lane, rc31 = st - 31;
-            if (st <= tfinal && rc31 >= 0 && rc31 <= span) ring[(start + rc31) & rmask] = ws->bout[st & 31];
+            if (st <= tfinal && rc31 >= 0 && rc31 <= span)
+                ring[(start + rc31) & rmask] =
+                    make_int4(ws->bout[0][st & 31], ws->bout[1][st & 31], ws->bout[2][st & 31], 0);
         }
         if constexpr (MODE == MODE_EXEC) {
             if ((tfinal % SPW) != SPW - 1) io.codes[wbase + (long long)(tfinal / SPW) * 32 + lane] = cw;
@@ -296,7 +315,7 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             if (__any_sync(FULL, upd)) bound_words = cum_words;
             upd = false;
         }
-        const int Wtail = ws->bout[tfinal & 31].z;
+        const int Wtail = ws->bout[2][tfinal & 31];
         if (e - start + 4 > rmask) {  // strip wider than the ring: the parked row has been overwritten
             flags |= SF_RING;
             break;

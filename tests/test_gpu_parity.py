@@ -142,3 +142,16 @@ def test_deterministic_repeat():
     g1, *_ = run_both(w.T, w.Q, w.seeds)
     g2, *_ = run_both(w.T, w.Q, w.seeds)
     assert np.array_equal(g1.rec, g2.rec) and g1.cigar == g2.cigar
+
+
+def test_unfolded_profile_large_scores():
+    """Scores too large to fold O+E into the int16 column profile (|sub + O + E| > 32767): the kernels take
+    the unfolded path (separate O+E add)."""
+    hox = np.array([[91, -114, -31, -123], [-114, 100, -125, -31], [-31, -125, 100, -114], [-123, -31, -114, 91]])
+    rng = random.Random(123)
+    T = rseq(rng, 3000)
+    Q = mutate(rng, T)
+    seeds = [(rng.randint(0, 3000), rng.randint(0, len(Q))) for _ in range(30)] + [(1500, 1500)]
+    bad, *_ = compare(T, Q, seeds, sub=hox * 200, gap_open=8000, gap_extend=600, ydrop=8000 + 300 * 600,
+                      gapped_threshold=600000)
+    assert_ok(bad)
