@@ -64,12 +64,10 @@ __device__ __forceinline__ int kill_fma(int s, int thr, int mOE, int one, int ze
 // predicated shared-memory store / load (keeps per-lane staging as predicated instructions, not a branch)
 __device__ __forceinline__ void st_shared_if(bool p, unsigned addr, int v) {
     asm volatile("{ .reg .pred q; setp.ne.u32 q, %0, 0; @q st.shared.b32 [%1], %2; }" ::"r"((unsigned)p), "r"(addr),
-                 "r"(v)
-                 : "memory");
+                 "r"(v));
 }
 __device__ __forceinline__ void ld_shared_if(bool p, unsigned addr, int& v) {
-    asm volatile("{ .reg .pred q; setp.ne.u32 q, %1, 0; @q ld.shared.b32 %0, [%2]; }" : "+r"(v) : "r"((unsigned)p), "r"(addr)
-                 : "memory");
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %1, 0; @q ld.shared.b32 %0, [%2]; }" : "+r"(v) : "r"((unsigned)p), "r"(addr));
 }
 
 __device__ __forceinline__ int prmt(int a, int b, int s) {

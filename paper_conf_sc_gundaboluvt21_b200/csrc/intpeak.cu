@@ -3,12 +3,22 @@
 // add-max VIADDMNMX), on every SM at full occupancy; reports lane-operations per second (one SASS integer
 // instruction on one lane = one op) and the SM clock observed through clock64().
 #include <cuda_runtime.h>
+#include <cstdio>
+#include <cstdlib>
+
 #include "internal.h"
 
 namespace fz {
 
+__device__ __forceinline__ unsigned long long gtimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+
 template <int KIND>
 __global__ void k_ipeak(int iters, int* out, int seed, long long* cycles) {
+    const unsigned long long g0 = gtimer();
     int a[8], x[8];
 #pragma unroll
     for (int k = 0; k < 8; ++k) {
@@ -28,11 +38,15 @@ __global__ void k_ipeak(int iters, int* out, int seed, long long* cycles) {
         }
     }
     const long long c1 = clock64();
+    const unsigned long long g1 = gtimer();
     int r = 0;
 #pragma unroll
     for (int k = 0; k < 8; ++k) r ^= a[k];
     if (r == 0x7fffffff) out[0] = r;
-    if (threadIdx.x == 0 && blockIdx.x == 0) *cycles = c1 - c0;
+    if (threadIdx.x == 0 && blockIdx.x == 0) {
+        cycles[0] = c1 - c0;
+        cycles[1] = (long long)(g1 - g0);
+    }
 }
 
 template <int KIND>
@@ -62,6 +76,7 @@ cudaError_t int_peak_run(int device, float target_ms, double* ops_per_s, double*
     if ((e = cudaMalloc(&out, 64)) != cudaSuccess) return e;
     if ((e = cudaMalloc(&cyc, 64)) != cudaSuccess) return e;
     double best = 0, best_mhz = 0;
+    const bool verbose = getenv("FASTZ_INTPEAK_VERBOSE") != nullptr;
     for (int kind = 0; kind < 3; ++kind) {
         int iters = 256;
         float ms = 0;
@@ -72,13 +87,18 @@ cudaError_t int_peak_run(int device, float target_ms, double* ops_per_s, double*
             if (ms >= target_ms) break;
             iters = (int)(iters * (ms > 0.05f ? 1.2f * target_ms / ms : 8.0f));
         }
-        long long c = 0;
-        cudaMemcpy(&c, cyc, sizeof(c), cudaMemcpyDeviceToHost);
+        long long c[2] = {0, 1};
+        cudaMemcpy(c, cyc, sizeof(c), cudaMemcpyDeviceToHost);
         const double ops = (double)sms * 8 * 256 * (double)iters * 16 * 8;
         const double rate = ops / (ms * 1e-3);
+        const double mhz_k = c[1] > 0 ? (double)c[0] / (double)c[1] * 1e3 : 0.0;  // cycles per ns -> MHz
+        if (verbose)
+            fprintf(stderr, "int_peak kind %d (%s): %.3f Tops/s, %.1f lane-ops/clk/SM at %.0f MHz\n", kind,
+                    kind == 0 ? "IMNMX" : (kind == 1 ? "IADD" : "VIADDMNMX"), rate / 1e12,
+                    mhz_k > 0 ? rate / (sms * mhz_k * 1e6) : 0.0, mhz_k);
         if (rate > best) {
             best = rate;
-            best_mhz = (double)c / (ms * 1e-3) / 1e6;
+            best_mhz = mhz_k;
         }
     }
     cudaFree(out);

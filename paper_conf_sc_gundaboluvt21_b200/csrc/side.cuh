@@ -98,7 +98,11 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
     const unsigned sb_in = (unsigned)__cvta_generic_to_shared(&ws->bin[0][0]);
     const unsigned sb_out = (unsigned)__cvta_generic_to_shared(&ws->bout[0][0]);
 
-    int start = 0, Wleft0 = NEG, lastlive = -1, Emax = -1, Wfar = NEG;
+    // W left of column 0 is V(i,-1) - Y = -inf; any value <= -Y gives the same thresholds (only the origin has
+    // no finite neighbour, and it is live for any threshold <= 0).  -(Y+1) keeps the cells that lanes compute
+    // before the strip's first column (ramp-up, left of column 0) dead, so ramp-up runs unchecked.
+    const int Wout = -P.Y - 1;
+    int start = 0, Wleft0 = Wout, lastlive = -1, Emax = -1, Wfar = NEG;
     int best = NEG + 1, bi = INT_MAX, bj = INT_MAX;
     long long cum_words = 0, bound_words = 0, cells = 0;
     uint32_t flags = 0;
@@ -280,9 +284,10 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
 #pragma unroll 1
                 for (int u = 0; u < 16; ++u)
                     if (step(yes, yes, t + u, u, u & 3, cbase)) { fin = true; break; }
-            } else if (t >= 32 && t + 15 <= span) {
-                // steady state: every lane valid for all 16 steps; 4-step unrolled body keeps the hot loop
-                // inside the instruction cache
+            } else if (t + 15 <= span) {
+                // steady state: no lane is past column N during these 16 steps (lanes still left of the strip's
+                // first column compute dead cells: all their inputs are dead and their threshold is >= -(Y+1));
+                // 4-step unrolled body keeps the hot loop inside the instruction cache
 #pragma unroll 1
                 for (int q = 0; q < 16 && !fin; q += 4) {
 #pragma unroll
