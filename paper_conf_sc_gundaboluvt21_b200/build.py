@@ -13,7 +13,7 @@ SOURCES = ["api.cu", "kernels.cu", "intpeak.cu"]
 HEADERS = ["dp.cuh", "side.cuh", "internal.h"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",
-         "-Xcompiler", "-fPIC", "-shared", "-Xptxas", "-warn-spills"]
+         "-Xcompiler", "-fPIC", "-shared", "-Xptxas", "-warn-spills", "-diag-suppress", "177"]
 
 
 def _stale() -> bool:

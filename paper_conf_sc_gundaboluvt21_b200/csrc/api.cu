@@ -50,7 +50,7 @@ struct fastz_ctx {
     DevParams dp{};
     int tlen = 0, qlen = 0;
     DBuf Tf, Tr, Qf, Qr, stage;
-    DBuf seeds, score, ti, qj, flags, eops, bound;
+    DBuf seeds, score, ti, qj, flags, eops, bound, maxsw, esc;
     DBuf woff, soff, roff, bin, list, counters, totals, tmpa, tmpb, tmpc, scan_tmp;
     DBuf codes, stab, runs, nruns, ciglen, cigar, recs, cells, ring, small;
     int R = 4, grid = 0, nslots = 0, rmask = 0;
@@ -182,6 +182,7 @@ SideArrays make_sides(fastz_ctx* c) {
     s.flags = P_<uint32_t>(c->flags);
     s.eops = P_<unsigned long long>(c->eops);
     s.bound = P_<long long>(c->bound);
+    s.maxsw = P_<int>(c->maxsw);
     return s;
 }
 
@@ -194,6 +195,7 @@ ExecPlan make_plan(fastz_ctx* c) {
     p.list = P_<int>(c->list);
     p.counters = P_<int>(c->counters);
     p.totals = P_<long long>(c->totals);
+    p.esc = P_<int>(c->esc);
     return p;
 }
 
@@ -256,7 +258,7 @@ void fastz_destroy(fastz_ctx* c) {
     cudaSetDevice(c->device);
     if (c->stream) cudaStreamSynchronize(c->stream);
     DBuf* bufs[] = {&c->Tf, &c->Tr, &c->Qf, &c->Qr, &c->stage, &c->seeds, &c->score, &c->ti, &c->qj,
-                    &c->flags, &c->eops, &c->bound, &c->woff, &c->soff, &c->roff, &c->bin, &c->list,
+                    &c->flags, &c->eops, &c->bound, &c->maxsw, &c->esc, &c->woff, &c->soff, &c->roff, &c->bin, &c->list,
                     &c->counters, &c->totals, &c->tmpa, &c->tmpb, &c->tmpc, &c->scan_tmp, &c->codes,
                     &c->stab, &c->runs, &c->nruns, &c->ciglen, &c->cigar, &c->recs, &c->cells, &c->ring,
                     &c->small};
@@ -351,6 +353,8 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     AL(flags, std::max<int64_t>(ns, 1) * 4);
     AL(eops, std::max<int64_t>(ns, 1) * 8);
     AL(bound, std::max<int64_t>(ns, 1) * 8);
+    AL(maxsw, std::max<int64_t>(ns, 1) * 4);
+    AL(esc, std::max<int64_t>(ns, 1) * 4);
     AL(woff, std::max<int64_t>(ns, 1) * 8);
     AL(soff, std::max<int64_t>(ns, 1) * 8);
     AL(roff, std::max<int64_t>(ns, 1) * 8);
@@ -381,8 +385,9 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
 
     SideArrays sa = make_sides(c);
     ExecPlan pl = make_plan(c);
-    int* counters = P_<int>(c->counters);
-    CK(launch_inspect(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, &counters[0], st));
+    const int esc = escalate_strips();
+    CK(launch_inspect(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, esc > 0 ? esc : INT_MAX, st));
+    if (esc > 0) CK(launch_inspect_block(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, st));
     CK(cudaEventRecord(c->ev[2], st));
     CK(launch_bin(c->R, sa, (int)ns, pl, c->scan_tmp.p, stb, P_<long long>(c->tmpa), P_<long long>(c->tmpb),
                   P_<long long>(c->tmpc), st));
@@ -390,7 +395,7 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
 
     // host sync 1: sizes of the executor's traceback pool
     struct {
-        long long totals[4];
+        long long totals[5];
         int counters[24];
         long long bad;
     } h;
@@ -402,11 +407,13 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     if (h.counters[20]) return fail(FASTZ_ERANGE, "an explored band is wider than the per-warp boundary ring");
     const long long words = h.totals[0], strips = h.totals[1], nrun = h.totals[2];
     c->nexec = h.totals[3];
+    const long long nblock = h.totals[4];
     AL(codes, std::max<long long>(words, 1) * 4);
     AL(stab, std::max<long long>(strips, 1) * 8);
     AL(runs, std::max<long long>(nrun, 1) * 4);
     Outputs o = make_out(c);
-    CK(launch_execute(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, (int)c->nexec, o, st));
+    CK(launch_execute(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, (int)c->nexec, (int)nblock, o,
+                      st));
     CK(cudaEventRecord(c->ev[4], st));
     CK(launch_traceback(c->R, sa, pl, (int)c->nexec, o, st));
     CK(cudaEventRecord(c->ev[5], st));

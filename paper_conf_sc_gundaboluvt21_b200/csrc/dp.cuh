@@ -33,7 +33,7 @@ constexpr int CP_RING = 128;      // column-profile ring entries per warp (+16 m
 constexpr int EAGER_W = 17;       // eager code window: rows/cols 0..16 (16x16)
 
 // side flags
-constexpr uint32_t SF_EAGER = 1u, SF_OVERFLOW = 2u, SF_RING = 4u, SF_EXEC_MISMATCH = 8u;
+constexpr uint32_t SF_EAGER = 1u, SF_OVERFLOW = 2u, SF_RING = 4u, SF_ESCALATE = 8u;
 
 struct DevParams {
     int cp[10];        // column profile per query base b (0..3) and the origin profile (b = 4):

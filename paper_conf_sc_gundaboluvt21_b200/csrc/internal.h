@@ -15,7 +15,8 @@ struct SideArrays {
     int* qj;             // j*
     uint32_t* flags;     // SF_* | eager op count << 8
     unsigned long long* eops;  // eager ops, 2 bits each, emission order (peak -> origin)
-    long long* bound;    // executor words bound (0 for eager sides)
+    long long* bound;    // executor words bound, compact layout (0 for eager sides)
+    int* maxsw;          // executor words of the widest strip up to the peak strip (block layout)
 };
 
 struct Batch {
@@ -31,9 +32,13 @@ struct ExecPlan {
     long long* soff;     // strip-table offset
     long long* roff;     // run-buffer offset
     int* bin;            // per side bin (0 = eager)
-    int* list;           // executor order: non-eager sides, larger bins first
-    int* counters;       // [0] inspector queue, [1] executor queue, [2..9] bin counts, [10..17] bin cursors
-    long long* totals;   // [0] words, [1] strips, [2] runs, [3] n_exec
+    int* list;           // executor order: non-eager sides, larger bins first; bins >= 3 (block per side)
+                         // occupy list[0, totals[4])
+    int* counters;       // [0] inspector queue, [1] executor warp queue, [2..8] bin counts, [10..16] bin cursors,
+                         // [20] ring overflow, [21] escalated sides, [22] block inspector queue,
+                         // [23] executor block queue
+    long long* totals;   // [0] words, [1] strips, [2] runs, [3] n_exec, [4] n_exec_block
+    int* esc;            // escalated sides (inspector -> block inspector)
 };
 
 struct Outputs {
@@ -54,7 +59,10 @@ cudaError_t launch_validate_seeds(const long long* seeds, int n, int tlen, int q
                                   cudaStream_t st);
 int inspector_blocks_per_sm(int R);
 cudaError_t launch_inspect(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
-                           const SideArrays& sa, int* counter, cudaStream_t st);
+                           const SideArrays& sa, const ExecPlan& pl, int budget, cudaStream_t st);
+cudaError_t launch_inspect_block(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
+                                 const SideArrays& sa, const ExecPlan& pl, cudaStream_t st);
+int escalate_strips();  // FASTZ_ESCALATE_STRIPS (default 16; 0 disables block-per-side inspection)
 cudaError_t launch_census(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
                           long long* cells, int* counter, cudaStream_t st);
 cudaError_t launch_bin(int R, const SideArrays& sa, int nsides, const ExecPlan& pl, void* scan_tmp,
@@ -62,7 +70,7 @@ cudaError_t launch_bin(int R, const SideArrays& sa, int nsides, const ExecPlan& 
                        cudaStream_t st);
 size_t scan_tmp_bytes(int n);
 cudaError_t launch_execute(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
-                           const SideArrays& sa, const ExecPlan& pl, int nexec, const Outputs& o,
+                           const SideArrays& sa, const ExecPlan& pl, int nexec, int nblock, const Outputs& o,
                            cudaStream_t st);
 cudaError_t launch_traceback(int R, const SideArrays& sa, const ExecPlan& pl, int nexec, const Outputs& o,
                              cudaStream_t st);

@@ -94,75 +94,133 @@ __device__ __forceinline__ void smem_init(SmemDP& sm, const DevParams& P) {
     __syncthreads();
 }
 
-// ------------------------------------------------------------------------------------------------- inspector
-// Persistent: each warp pops one-sided extensions from an atomic queue (load balance replaces the paper's
-// 32 CUDA streams, P:218).  Score-only DP + eager 17x17 corner codes; when the peak lies inside the
-// eager window the warp's lane 0 walks the codes at once (P:166-170) and the side skips the executor.
-template <int R, bool FOLD>
-__global__ void __launch_bounds__(WARPS * 32) k_inspect(DevParams P, Batch b, int4* ring, int rmask,
-                                                         SideArrays sa, int* counter) {
-    __shared__ SmemDP sm;
-    smem_init(sm, P);
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    SideIO io;
-    io.ring = ring + (size_t)(blockIdx.x * WARPS + warp) * (size_t)(rmask + 1);
+__device__ __forceinline__ void io_init(SideIO& io, SmemDP& sm, int4* ring, int rmask, int warp_slot, int warp) {
+    io.ring = ring + (size_t)warp_slot * (size_t)(rmask + 1);
     io.rmask = rmask;
     io.ws = &sm.w[warp];
     io.cptab = sm.cptab;
     io.ecodes = sm.ecodes[warp];
-    io.eager_max = P.eager_max;
+    io.eager_max = -1;
     io.codes = nullptr;
     io.stab = nullptr;
+    io.budget = INT_MAX;
+    io.ps = nullptr;
+    io.wi = warp;
+    io.K = WARPS;
+    io.maxsw = 0;
+}
+
+// eager traceback by lane 0 over the 17x17 corner codes; returns ops (2 bits each, peak -> origin)
+__device__ __forceinline__ unsigned long long eager_walk(const uint8_t* ec, int i, int j, int& nops) {
+    unsigned long long ops = 0;
+    nops = 0;
+    int state = 0;
+    while (i > 0 || j > 0) {
+        const uint32_t code = ec[i * EAGER_W + j];
+        if (state == 0) {
+            const uint32_t src = code & 3u;
+            if (src == 0) {
+                ops |= (unsigned long long)OP_M << (2 * nops);
+                ++nops; --i; --j;
+                continue;
+            }
+            state = (int)src;
+        }
+        if (state == 1) {
+            ops |= (unsigned long long)OP_D << (2 * nops);
+            ++nops;
+            state = (code >> 2) & 1u ? 1 : 0;
+            --i;
+        } else {
+            ops |= (unsigned long long)OP_I << (2 * nops);
+            ++nops;
+            state = (code >> 3) & 1u ? 2 : 0;
+            --j;
+        }
+    }
+    return ops;
+}
+
+__device__ __forceinline__ void write_side(const DevParams& P, const SideArrays& sa, int side, const SideOut& o,
+                                           uint32_t flags, unsigned long long ops, int nops) {
+    sa.score[side] = o.best + P.OE;
+    sa.ti[side] = o.bi;
+    sa.qj[side] = o.bj;
+    sa.flags[side] = flags | ((uint32_t)nops << 8);
+    sa.eops[side] = ops;
+    sa.bound[side] = (flags & SF_EAGER) ? 0 : o.bound_words;
+    sa.maxsw[side] = (flags & SF_EAGER) ? 0 : o.bound_maxsw;
+}
+
+// ------------------------------------------------------------------------------------------------- inspector
+// Persistent: each warp pops one-sided extensions from an atomic queue (load balance replaces the paper's
+// 32 CUDA streams, P:218).  Score-only DP + eager 17x17 corner codes; when the peak lies inside the
+// eager window the warp's lane 0 walks the codes at once (P:166-170) and the side skips the executor.
+// A side still running after `budget` strips is handed to the block-per-side inspector (escalation).
+template <int R, bool FOLD>
+__global__ void __launch_bounds__(WARPS * 32) k_inspect(DevParams P, Batch b, int4* ring, int rmask,
+                                                         SideArrays sa, ExecPlan pl, int budget) {
+    __shared__ SmemDP sm;
+    smem_init(sm, P);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    SideIO io;
+    io_init(io, sm, ring, rmask, blockIdx.x * WARPS + warp, warp);
+    io.eager_max = P.eager_max;
+    io.budget = budget;
     const int nsides = 2 * b.nseeds;
     for (;;) {
         int side = 0;
-        if (lane == 0) side = atomicAdd(counter, 1);
+        if (lane == 0) side = atomicAdd(&pl.counters[0], 1);
         side = __shfl_sync(FULL, side, 0);
         if (side >= nsides) break;
         setup_side(b, side, io);
         SideOut o;
-        run_side<R, MODE_INSPECT, true, FOLD>(P, io, o);
+        run_side<R, MODE_INSPECT, true, FOLD, false>(P, io, o);
         __syncwarp();  // eager corner codes (shared memory) written by lanes 0..4 -> read by lane 0
         if (lane == 0) {
-            uint32_t flags = o.flags;
-            unsigned long long ops = 0;
-            int nops = 0;
-            const bool eager = o.bi <= P.eager_max && o.bj <= P.eager_max && !(flags & (SF_RING | SF_OVERFLOW));
-            if (eager) {
-                int i = o.bi, j = o.bj, state = 0;
-                while (i > 0 || j > 0) {
-                    const uint32_t code = io.ecodes[i * EAGER_W + j];
-                    if (state == 0) {
-                        const uint32_t src = code & 3u;
-                        if (src == 0) {
-                            ops |= (unsigned long long)OP_M << (2 * nops);
-                            ++nops; --i; --j;
-                            continue;
-                        }
-                        state = (int)src;
-                    }
-                    if (state == 1) {
-                        ops |= (unsigned long long)OP_D << (2 * nops);
-                        ++nops;
-                        state = (code >> 2) & 1u ? 1 : 0;
-                        --i;
-                    } else {
-                        ops |= (unsigned long long)OP_I << (2 * nops);
-                        ++nops;
-                        state = (code >> 3) & 1u ? 2 : 0;
-                        --j;
-                    }
+            if (o.flags & SF_ESCALATE) {
+                pl.esc[atomicAdd(&pl.counters[21], 1)] = side;
+            } else {
+                uint32_t flags = o.flags;
+                unsigned long long ops = 0;
+                int nops = 0;
+                if (o.bi <= P.eager_max && o.bj <= P.eager_max && !(flags & (SF_RING | SF_OVERFLOW))) {
+                    ops = eager_walk(io.ecodes, o.bi, o.bj, nops);
+                    flags |= SF_EAGER;
                 }
-                flags |= SF_EAGER;
+                write_side(P, sa, side, o, flags, ops, nops);
             }
-            sa.score[side] = o.best + P.OE;
-            sa.ti[side] = o.bi;
-            sa.qj[side] = o.bj;
-            sa.flags[side] = flags | ((uint32_t)nops << 8);
-            sa.eops[side] = ops;
-            sa.bound[side] = eager ? 0 : o.bound_words;
         }
         __syncwarp();
+    }
+}
+
+// Block per side (long sides, escalated by k_inspect): the CTA's warps pipeline the side's strips.
+template <int R, bool FOLD>
+__global__ void __launch_bounds__(WARPS * 32) k_inspect_block(DevParams P, Batch b, int4* ring, int rmask,
+                                                               SideArrays sa, ExecPlan pl) {
+    __shared__ SmemDP sm;
+    __shared__ PipeShared ps;
+    __shared__ int cur;
+    smem_init(sm, P);
+    const int warp = threadIdx.x >> 5;
+    for (;;) {
+        if (threadIdx.x == 0) {
+            const int i = atomicAdd(&pl.counters[22], 1);
+            cur = i < pl.counters[21] ? pl.esc[i] : -1;
+            pipe_reset(&ps);
+        }
+        __syncthreads();
+        const int side = cur;
+        if (side < 0) break;
+        SideIO io;
+        io_init(io, sm, ring, rmask, blockIdx.x * WARPS, warp);
+        io.ps = &ps;
+        setup_side(b, side, io);
+        SideOut o;
+        run_side<R, MODE_INSPECT, false, FOLD, true>(P, io, o);
+        if (threadIdx.x == 0) write_side(P, sa, side, o, o.flags, 0ull, 0);
+        __syncthreads();
     }
 }
 
@@ -173,14 +231,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int
     smem_init(sm, P);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     SideIO io;
-    io.ring = ring + (size_t)(blockIdx.x * WARPS + warp) * (size_t)(rmask + 1);
-    io.rmask = rmask;
-    io.ws = &sm.w[warp];
-    io.cptab = sm.cptab;
-    io.ecodes = nullptr;
-    io.eager_max = -1;
-    io.codes = nullptr;
-    io.stab = nullptr;
+    io_init(io, sm, ring, rmask, blockIdx.x * WARPS + warp, warp);
     const int nsides = 2 * b.nseeds;
     for (;;) {
         int side = 0;
@@ -189,31 +240,53 @@ __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int
         if (side >= nsides) break;
         setup_side(b, side, io);
         SideOut o;
-        run_side<R, MODE_CENSUS, false, FOLD>(P, io, o);
+        run_side<R, MODE_CENSUS, false, FOLD, false>(P, io, o);
         if (lane == 0) cells[side] = (o.flags & SF_RING) ? -1 : o.cells;
         __syncwarp();
     }
 }
 
 // ------------------------------------------------------------------------------------------------- executor
-// Trimmed executor: the DP over [0,i*]x[0,j*] only, writing traceback codes.  Persistent warps
-// pop non-eager sides in bin order, largest bins first (length binning P:209-211 used as an LPT schedule).
+// Trimmed executor: the DP over [0,i*]x[0,j*] only, writing traceback codes.  Length binning
+// as a schedule: the CTAs first take the long sides (bins >= 3, block per side, strips pipelined
+// across the CTA's warps), then every warp takes short sides (bins 1-2, warp per side), larger bins first.
 template <int R, bool FOLD>
 __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, int4* ring, int rmask,
-                                                         SideArrays sa, ExecPlan pl, int nexec, Outputs out) {
+                                                         SideArrays sa, ExecPlan pl, int nexec, int nblock,
+                                                         Outputs out) {
     __shared__ SmemDP sm;
+    __shared__ PipeShared ps;
+    __shared__ int cur;
     smem_init(sm, P);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    for (;;) {  // block phase
+        if (threadIdx.x == 0) {
+            const int i = atomicAdd(&pl.counters[23], 1);
+            cur = i < nblock ? pl.list[i] : -1;
+            pipe_reset(&ps);
+        }
+        __syncthreads();
+        const int side = cur;
+        if (side < 0) break;
+        SideIO io;
+        io_init(io, sm, ring, rmask, blockIdx.x * WARPS, warp);
+        io.ps = &ps;
+        setup_side(b, side, io);
+        io.M = sa.ti[side];
+        io.N = sa.qj[side];
+        io.codes = out.codes + pl.woff[side];
+        io.stab = out.stab + pl.soff[side];
+        io.maxsw = sa.maxsw[side];
+        SideOut o;
+        run_side<R, MODE_EXEC, false, FOLD, true>(P, io, o);
+        if (threadIdx.x == 0 && (o.flags & SF_RING)) atomicOr(&sa.flags[side], SF_RING);
+        __syncthreads();
+    }
     SideIO io;
-    io.ring = ring + (size_t)(blockIdx.x * WARPS + warp) * (size_t)(rmask + 1);
-    io.rmask = rmask;
-    io.ws = &sm.w[warp];
-    io.cptab = sm.cptab;
-    io.ecodes = nullptr;
-    io.eager_max = -1;
-    for (;;) {
+    io_init(io, sm, ring, rmask, blockIdx.x * WARPS + warp, warp);
+    for (;;) {  // warp phase
         int idx = 0;
-        if (lane == 0) idx = atomicAdd(&pl.counters[1], 1);
+        if (lane == 0) idx = nblock + atomicAdd(&pl.counters[1], 1);
         idx = __shfl_sync(FULL, idx, 0);
         if (idx >= nexec) break;
         const int side = pl.list[idx];
@@ -223,7 +296,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, in
         io.codes = out.codes + pl.woff[side];
         io.stab = out.stab + pl.soff[side];
         SideOut o;
-        run_side<R, MODE_EXEC, false, FOLD>(P, io, o);
+        run_side<R, MODE_EXEC, false, FOLD, false>(P, io, o);
         if (lane == 0 && (o.flags & SF_RING)) atomicOr(&sa.flags[side], SF_RING);
         __syncwarp();
     }
@@ -294,27 +367,31 @@ __device__ __forceinline__ int bin_of(int m) {
 
 template <int R>
 __global__ void k_bin_count(SideArrays sa, int nsides, ExecPlan pl, long long* words, long long* strips,
-                            long long* runs) {
+                            long long* runs, int bblock) {
     const int s = blockIdx.x * blockDim.x + threadIdx.x;
     if (s >= nsides) return;
-    const bool eager = sa.flags[s] & SF_EAGER;
+    const uint32_t fl = sa.flags[s];
+    const bool eager = fl & SF_EAGER;
     const int ti = sa.ti[s], qj = sa.qj[s];
     const int bin = eager ? 0 : bin_of(ti > qj ? ti : qj);
     pl.bin[s] = bin;
     atomicAdd(&pl.counters[2 + bin], 1);
-    if (sa.flags[s] & SF_RING) atomicOr(&pl.counters[20], 1);
-    words[s] = eager ? 0 : sa.bound[s];
-    strips[s] = eager ? 0 : ti / (32 * R) + 1;
+    if (fl & SF_RING) atomicOr(&pl.counters[20], 1);
+    const long long ns = ti / (32 * R) + 1;
+    // bins >= 3 run block per side: strip s of the side owns words [s * maxsw, (s + 1) * maxsw)
+    words[s] = eager ? 0 : (bin >= bblock ? ns * (long long)sa.maxsw[s] : sa.bound[s]);
+    strips[s] = eager ? 0 : ns;
     runs[s] = eager ? 0 : (long long)ti + qj + 1;
 }
 
 __global__ void k_bin_offsets(ExecPlan pl, int nsides, const long long* words, const long long* strips,
-                              const long long* runs) {
+                              const long long* runs, int bblock) {
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
-    int run = 0;
+    int run = 0, nblock = 0;
     for (int bin = 6; bin >= 1; --bin) {  // larger bins first
         pl.counters[10 + bin] = run;
         run += pl.counters[2 + bin];
+        if (bin == bblock) nblock = run;
     }
     if (nsides > 0) {
         pl.totals[0] = pl.woff[nsides - 1] + words[nsides - 1];
@@ -324,6 +401,7 @@ __global__ void k_bin_offsets(ExecPlan pl, int nsides, const long long* words, c
         pl.totals[0] = pl.totals[1] = pl.totals[2] = 0;
     }
     pl.totals[3] = run;
+    pl.totals[4] = nblock;
 }
 
 __global__ void k_bin_scatter(ExecPlan pl, int nsides) {
@@ -335,6 +413,12 @@ __global__ void k_bin_scatter(ExecPlan pl, int nsides) {
     pl.list[pos] = s;
 }
 
+int block_bin() {  // smallest executor bin run block per side (FASTZ_BLOCK_BIN, default 3: > 2048)
+    const char* e = getenv("FASTZ_BLOCK_BIN");
+    int v = e ? atoi(e) : 3;
+    return v < 1 ? 1 : (v > 7 ? 7 : v);
+}
+
 size_t scan_tmp_bytes(int n) {
     size_t bytes = 0;
     cub::DeviceScan::ExclusiveSum(nullptr, bytes, (const long long*)nullptr, (long long*)nullptr, n > 0 ? n : 1);
@@ -343,11 +427,12 @@ size_t scan_tmp_bytes(int n) {
 
 cudaError_t launch_bin(int R, const SideArrays& sa, int nsides, const ExecPlan& pl, void* tmp, size_t tmp_bytes,
                        long long* words, long long* strips, long long* runs, cudaStream_t st) {
+    const int bb = block_bin();
     if (nsides > 0) {
         const int g = (nsides + 255) / 256;
         switch (R) {
-            case 2: k_bin_count<2><<<g, 256, 0, st>>>(sa, nsides, pl, words, strips, runs); break;
-            default: k_bin_count<4><<<g, 256, 0, st>>>(sa, nsides, pl, words, strips, runs); break;
+            case 2: k_bin_count<2><<<g, 256, 0, st>>>(sa, nsides, pl, words, strips, runs, bb); break;
+            default: k_bin_count<4><<<g, 256, 0, st>>>(sa, nsides, pl, words, strips, runs, bb); break;
         }
         cudaError_t e;
         size_t b = tmp_bytes;
@@ -357,7 +442,7 @@ cudaError_t launch_bin(int R, const SideArrays& sa, int nsides, const ExecPlan& 
         b = tmp_bytes;
         if ((e = cub::DeviceScan::ExclusiveSum(tmp, b, runs, pl.roff, nsides, st)) != cudaSuccess) return e;
     }
-    k_bin_offsets<<<1, 1, 0, st>>>(pl, nsides, words, strips, runs);
+    k_bin_offsets<<<1, 1, 0, st>>>(pl, nsides, words, strips, runs, bb);
     if (nsides > 0) k_bin_scatter<<<(nsides + 255) / 256, 256, 0, st>>>(pl, nsides);
     return cudaGetLastError();
 }
@@ -466,8 +551,12 @@ __global__ void k_combine_write(DevParams P, Batch b, SideArrays sa, ExecPlan pl
     a.right_score = sa.score[Rt];
     a.score = a.left_score + a.right_score;
     const uint32_t fl = sa.flags[L], fr = sa.flags[Rt];
-    a.flags = (a.score >= P.K ? FASTZ_FLAG_ABOVE_K : 0u) | ((fl & SF_EAGER) ? FASTZ_FLAG_LEFT_EAGER : 0u) |
-              ((fr & SF_EAGER) ? FASTZ_FLAG_RIGHT_EAGER : 0u) |
+    // eager classification: peak inside the eager window (escalated sides are traced back by the
+    // executor even then; the flag reports the classification)
+    const bool el = sa.ti[L] <= P.eager_max && sa.qj[L] <= P.eager_max;
+    const bool er = sa.ti[Rt] <= P.eager_max && sa.qj[Rt] <= P.eager_max;
+    a.flags = (a.score >= P.K ? FASTZ_FLAG_ABOVE_K : 0u) | (el ? FASTZ_FLAG_LEFT_EAGER : 0u) |
+              (er ? FASTZ_FLAG_RIGHT_EAGER : 0u) |
               (((fl | fr) & SF_OVERFLOW) ? FASTZ_FLAG_OVERFLOW : 0u);
     a.t_start = tpos - sa.ti[L];
     a.t_end = tpos + sa.ti[Rt];
@@ -487,14 +576,10 @@ cudaError_t launch_combine_write(const DevParams& P, const Batch& b, const SideA
 }
 
 // ------------------------------------------------------------------------------------------------- launchers
-int pick_R() {
-    static int r = 0;
-    if (!r) {
-        const char* e = getenv("FASTZ_R");
-        r = e ? atoi(e) : 4;
-        if (r != 2 && r != 4) r = 4;
-    }
-    return r;
+int pick_R() {  // read at fastz_create
+    const char* e = getenv("FASTZ_R");
+    const int r = e ? atoi(e) : 4;
+    return (r == 2 || r == 4) ? r : 4;
 }
 
 template <int R>
@@ -517,10 +602,25 @@ int inspector_blocks_per_sm(int R) { return R == 2 ? bps_of<2>() : bps_of<4>(); 
         }                                                                                \
     } while (0)
 
+int escalate_strips() {  // read per call: tests and ablations switch it at run time
+    const char* e = getenv("FASTZ_ESCALATE_STRIPS");
+    int v = e ? atoi(e) : 16;
+    return v < 0 ? 0 : v;
+}
+
+
+
 cudaError_t launch_inspect(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
-                           const SideArrays& sa, int* counter, cudaStream_t st) {
+                           const SideArrays& sa, const ExecPlan& pl, int budget, cudaStream_t st) {
     if (b.nseeds == 0) return cudaSuccess;
-    FZ_DISPATCH(k_inspect, grid, P, b, ring, rmask, sa, counter);
+    FZ_DISPATCH(k_inspect, grid, P, b, ring, rmask, sa, pl, budget);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_inspect_block(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
+                                 const SideArrays& sa, const ExecPlan& pl, cudaStream_t st) {
+    if (b.nseeds == 0) return cudaSuccess;
+    FZ_DISPATCH(k_inspect_block, grid, P, b, ring, rmask, sa, pl);
     return cudaGetLastError();
 }
 
@@ -532,9 +632,10 @@ cudaError_t launch_census(int R, int grid, const DevParams& P, const Batch& b, i
 }
 
 cudaError_t launch_execute(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
-                           const SideArrays& sa, const ExecPlan& pl, int nexec, const Outputs& o, cudaStream_t st) {
+                           const SideArrays& sa, const ExecPlan& pl, int nexec, int nblock, const Outputs& o,
+                           cudaStream_t st) {
     if (nexec == 0) return cudaSuccess;
-    FZ_DISPATCH(k_execute, grid, P, b, ring, rmask, sa, pl, nexec, o);
+    FZ_DISPATCH(k_execute, grid, P, b, ring, rmask, sa, pl, nexec, nblock, o);
     return cudaGetLastError();
 }
 

@@ -1,21 +1,31 @@
-// side.cuh -- one warp runs one one-sided extension, strip by strip (see dp.cuh for the layout).
+// side.cuh -- the strip engine: one one-sided extension, strip by strip (see dp.cuh for the cell math).
 //
-// MODE_INSPECT: score-only pass that finds the peak ("lightweight inspector"), records the 17x17 corner
-//               codes during the first steps of strip 0 for eager traceback, and bounds the
-//               executor's traceback storage (the executor's allocation is sized by the inspector).
-// MODE_EXEC:    the trimmed executor: the same DP restricted to [0,i*]x[0,j*] (exact, because the cone
-//               rule of reading R3 only looks inside the rectangle), writing 4-bit codes to HBM in a
-//               step-major layout: word (t / SPW) * 32 + lane of the strip holds lane's R rows for SPW steps,
-//               so each warp store is one coalesced 128-byte line (P:180's consolidation, done in registers).
-// MODE_CENSUS:  counts explored cells (origin + cells with a live diagonal/up/left neighbour), the GCUPS
-//               numerator; not on the timed path.
+// Two schedules of the same sweep:
+//  * SOLO (warp per problem): one warp runs strips 0, 1, 2, ... of a side.
+//  * PIPE (block per problem, long sides): the K warps of a CTA run strips s = w, w+K, w+2K, ... of ONE side
+//    concurrently; strip s consumes strip s-1's bottom row through the shared boundary ring as soon as it is
+//    flushed (progress flags in shared memory), so a long side advances K strips at a time.  Every
+//    synchronisation point (strip start, boundary loads, termination, strip finish) waits only on strip s-1,
+//    which is why the result is identical to SOLO (the cone rule of reading R3 is local).
+//
+// Modes:
+//  MODE_INSPECT: score-only pass that finds the peak ("lightweight inspector"), records the 17x17 corner
+//                codes during the first steps of strip 0 for eager traceback, and bounds the
+//                executor's traceback storage (the executor's allocation is sized by the inspector).
+//  MODE_EXEC:    the trimmed executor: the same DP restricted to [0,i*]x[0,j*] (exact, because the
+//                cone rule only looks inside the rectangle), writing 4-bit codes to HBM in a step-major
+//                layout: word (t / SPW) * 32 + lane of a strip holds lane's R rows for SPW steps, so each warp
+//                store is one coalesced 128-byte line (P:180's consolidation, done in registers).
+//  MODE_CENSUS:  counts explored cells (origin + cells with a live diagonal/up/left neighbour), the GCUPS
+//                numerator; not on the timed path.
 //
 // Per-step data movement (the paper's register exchange, re-designed for sm_100a):
 //  * lane l receives the bottom row (X, D, W) of lane l-1 with a ROTATING shuffle (src = l-1 mod 32): lane 0
 //    receives from lane 31, which -- after parking its own bottom row in shared staging -- holds the previous
 //    strip's boundary value for lane 0's next column.  No per-step global memory access, no lane-0 selects.
 //  * every 16 steps the warp moves 16 boundary values global ring -> shared staging (prefetched one block
-//    ahead) and 16 parked bottom-row values shared -> global ring, both coalesced.
+//    ahead) and 16 parked bottom-row values shared -> global ring, both coalesced; the parked values also
+//    give the bottom row's first/last live column (next strip's start, termination test).
 //  * termination: each lane keeps the last step at which one of its R cells was live; the strip is done at
 //    column x (lane 31's) iff no lane has had a live cell since it processed x and the boundary row has no
 //    live cell at or after x -- the unrolled form of the per-lane "done" chain (lane l is done at x iff its
@@ -29,10 +39,29 @@ namespace fz {
 
 enum { MODE_INSPECT = 0, MODE_EXEC = 1, MODE_CENSUS = 2 };
 
+constexpr int PIPE_SLOTS = 8;  // 2K slots for K = 4 warps: a slot is reused only after its consumer finished
+
 struct WarpSmem {
     int2 cp[CP_RING + 16];  // column profiles, ring over relative columns (+16 mirrored)
     int bin[3][32];         // boundary row staging (X, D, W; lane 0's input, served through lane 31)
     int bout[3][32];        // lane 31's bottom-row outputs (X, D, W) awaiting the global ring
+};
+
+// Block-per-problem (PIPE) shared state of one side.  Strip s owns slot s % PIPE_SLOTS.
+struct PipeShared {
+    volatile int sid[PIPE_SLOTS];    // strip id whose start/progress the slot currently describes
+    volatile int start[PIPE_SLOTS];  // strip start column
+    volatile int wleft[PIPE_SLOTS];  // W(top-1, start-1) of the strip
+    volatile int prog[PIPE_SLOTS];   // last bottom-row column flushed to the ring
+    volatile int first[PIPE_SLOTS];  // first live bottom-row column flushed so far (INT_MAX: none yet)
+    volatile int last[PIPE_SLOTS];   // last live bottom-row column flushed so far
+    volatile int done[PIPE_SLOTS];   // strip id whose finish (tail update, side state) is complete
+    volatile int end_strip;          // strip that ended the side (INT_MAX while running)
+    volatile int Emax, Wfar;         // boundary-ring state after the last finished strip
+    volatile unsigned flags;
+    volatile long long cum_words, bound_words;
+    volatile int maxsw, bound_maxsw;
+    int best[8], bi[8], bj[8];       // per-warp peaks for the final reduction
 };
 
 struct SideIO {
@@ -43,7 +72,7 @@ struct SideIO {
     int64_t Boff;
     int Bmax;                           // real query length (bases beyond are never read)
     int N;                              // columns 0..N (N <= Bmax; the executor trims to j*)
-    int4* __restrict__ ring;            // per-warp boundary ring, rmask + 1 entries {X, D, W, -}
+    int4* __restrict__ ring;            // boundary ring (per warp in SOLO, per CTA in PIPE), rmask + 1 entries
     int rmask;
     WarpSmem* ws;                       // shared staging of this warp
     const int2* cptab;                  // shared: 5 profiles (query base 0..3, zero)
@@ -51,12 +80,17 @@ struct SideIO {
     int eager_max;
     uint32_t* __restrict__ codes;       // executor: the side's code words
     int2* __restrict__ stab;            // executor: per strip {start column, word offset}
+    int budget;                         // SOLO inspector: strips before escalation to PIPE (INT_MAX: none)
+    PipeShared* ps;                     // PIPE: shared side state
+    int wi, K;                          // PIPE: warp index in the CTA, warps per side
+    int maxsw;                          // PIPE executor: words reserved per strip (from the inspector)
 };
 
 struct SideOut {
     int best, bi, bj;        // peak in X space (score = best + O + E), ties: min i, min j
     uint32_t flags;
-    long long bound_words;   // inspector: executor words up to the peak strip
+    long long bound_words;   // inspector: executor words up to the peak strip (compact layout)
+    int bound_maxsw;         // inspector: max words of one strip up to the peak strip (block layout)
     long long cells;         // census: explored cells (warp total)
     long long words;         // executor: words written
 };
@@ -78,11 +112,17 @@ __device__ __forceinline__ void cp_store(const SideIO& io, int rc, int code) {
     if (idx < 16) io.ws->cp[idx + CP_RING] = v;
 }
 
-__device__ __forceinline__ int4 boundary(const int4* __restrict__ ring, int rmask, int c, int Emax, int Wfar) {
-    return c <= Emax ? ring[c & rmask] : make_int4(NEG, NEG, Wfar, 0);
+// Boundary row value at column c: the ring holds exact entries up to column lim, beyond it the row is dead
+// with W = Wfar (reading R3: V beyond the last scanned column).  PIPE reads bypass L1 (written by other warps).
+template <bool PIPE>
+__device__ __forceinline__ int4 boundary(const int4* __restrict__ ring, int rmask, int c, int lim, int Wfar) {
+    if (c <= lim) return PIPE ? __ldcg(ring + (c & rmask)) : ring[c & rmask];
+    return make_int4(NEG, NEG, Wfar, 0);
 }
 
-template <int R, int MODE, bool EAGER, bool FOLD>
+__device__ __forceinline__ void pipe_wait() { __nanosleep(100); }
+
+template <int R, int MODE, bool EAGER, bool FOLD, bool PIPE>
 __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, SideOut& out) {
     constexpr int H = StripGeom<R>::H;
     constexpr int SPW = StripGeom<R>::SPW;
@@ -94,6 +134,7 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
     const int rmask = io.rmask;
     int4* __restrict__ ring = io.ring;
     WarpSmem* __restrict__ ws = io.ws;
+    PipeShared* __restrict__ ps = io.ps;
     const bool is31 = lane == 31;
     const unsigned sb_in = (unsigned)__cvta_generic_to_shared(&ws->bin[0][0]);
     const unsigned sb_out = (unsigned)__cvta_generic_to_shared(&ws->bout[0][0]);
@@ -102,14 +143,60 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
     // no finite neighbour, and it is live for any threshold <= 0).  -(Y+1) keeps the cells that lanes compute
     // before the strip's first column (ramp-up, left of column 0) dead, so ramp-up runs unchecked.
     const int Wout = -P.Y - 1;
-    int start = 0, Wleft0 = Wout, lastlive = -1, Emax = -1, Wfar = NEG;
+    // SOLO side state (registers); PIPE keeps it in *ps
+    int start = 0, Wleft0 = Wout, lastlive = -1, Emax = -1, Wfar = NEG, nfirst = INT_MAX;
     int best = NEG + 1, bi = INT_MAX, bj = INT_MAX;
     long long cum_words = 0, bound_words = 0, cells = 0;
+    int maxsw = 0, bound_maxsw = 0;
     uint32_t flags = 0;
     bool upd = false;
 
-    int s = 0;
-    for (int top = 0; top <= M; top += H, ++s) {
+    for (int s = PIPE ? io.wi : 0;; s += PIPE ? io.K : 1) {
+        const int slot = s % PIPE_SLOTS, pslot = (s + PIPE_SLOTS - 1) % PIPE_SLOTS;
+        // ------------------------------------------------------------------ strip start
+        if constexpr (PIPE) {
+            if (s * H > M) goto side_done;  // strip s-1 holds row M and ends the side: never start past it
+            if (s == 0) {
+                start = 0;
+                Wleft0 = Wout;
+            } else {
+                // wait until strip s-1 has flushed its first live bottom cell, or has finished
+                for (;;) {
+                    if (ps->end_strip < s) goto side_done;
+                    if (ps->sid[pslot] == s - 1) {
+                        const int f = ps->first[pslot];
+                        if ((f != INT_MAX && ps->prog[pslot] >= f) || ps->done[pslot] == s - 1) break;
+                    }
+                    pipe_wait();
+                }
+                __threadfence_block();
+                if (ps->end_strip < s) goto side_done;
+                start = ps->first[pslot];
+                const int sp = ps->start[pslot];
+                Wleft0 = start > sp ? __ldcg(ring + ((start - 1) & rmask)).z : ps->wleft[pslot];
+            }
+            __syncwarp();
+            if (lane == 0) {
+                ps->start[slot] = start;
+                ps->wleft[slot] = Wleft0;
+                ps->first[slot] = INT_MAX;
+                ps->last[slot] = -1;
+                ps->prog[slot] = start - 1;
+                __threadfence_block();
+                ps->sid[slot] = s;
+            }
+        } else {
+            if (s > 0) {
+                if (io.budget != INT_MAX && s >= io.budget) {  // long side: hand over to the block kernel
+                    flags |= SF_ESCALATE;
+                    break;
+                }
+                if (nfirst > start) Wleft0 = ring[(nfirst - 1) & rmask].z;
+                start = nfirst;
+            }
+        }
+        const int top = s * H;
+
         // ------------------------------------------------------------------ strip set-up
         int sel[R], X[R], I[R], W[R];
         const int r0 = top + lane * R;
@@ -129,22 +216,54 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         int xb = NEG, db = NEG, wb = NEG;
         const int span = N - start;
         const int tlast = span + 31;
-        const long long wbase = cum_words;  // executor: this strip's first word (relative to the side)
+        const long long wbase = PIPE ? (long long)s * io.maxsw : cum_words;  // executor: strip's first word
         if constexpr (MODE == MODE_EXEC) {
             if (lane == 0) io.stab[s] = make_int2(start, (int)wbase);
         }
+        // boundary source: SOLO -> ring up to Emax; PIPE -> ring up to strip s-1's progress, or (once it has
+        // finished) up to the side's Emax
+        int blim = Emax, bwf = Wfar;
+        bool pdone = !PIPE || s == 0;
+        auto pipe_sync = [&](int chi) {  // PIPE: make boundary columns <= chi readable
+            if constexpr (PIPE) {
+                if (s == 0) {
+                    blim = -1;
+                    bwf = NEG;
+                    return;
+                }
+                if (!pdone) {
+                    for (;;) {
+                        if (ps->done[pslot] == s - 1) {
+                            __threadfence_block();
+                            pdone = true;
+                            blim = ps->Emax;
+                            bwf = ps->Wfar;
+                            break;
+                        }
+                        const int pg = ps->prog[pslot];
+                        if (pg >= chi) {
+                            __threadfence_block();
+                            blim = pg;
+                            break;
+                        }
+                        pipe_wait();
+                    }
+                }
+            }
+        };
+        pipe_sync(start + 47);
         // staging: boundary for relative columns [0, 32), column profiles [0, 32); prefetch the next 16
         {
-            const int4 v = boundary(ring, rmask, start + lane, Emax, Wfar);
+            const int4 v = boundary<PIPE>(ring, rmask, start + lane, blim, bwf);
             ws->bin[0][lane] = v.x;
             ws->bin[1][lane] = v.y;
             ws->bin[2][lane] = v.z;
         }
         cp_store(io, lane, query_code(io, start + lane));
-        int4 bpre = make_int4(NEG, NEG, Wfar, 0);
+        int4 bpre = make_int4(NEG, NEG, bwf, 0);
         int qpre = 4;
         if (lane < 16) {
-            bpre = boundary(ring, rmask, start + 32 + lane, Emax, Wfar);
+            bpre = boundary<PIPE>(ring, rmask, start + 32 + lane, blim, bwf);
             qpre = query_code(io, start + 32 + lane);
         }
         __syncwarp();
@@ -154,8 +273,39 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             wb = ws->bin[2][0];
         }
         uint32_t cw = 0;
-        int lastlive_t = -1;   // last step at which this lane had a live cell (termination, see header)
+        int lastlive_t = -1;  // last step at which this lane had a live cell (termination, see header)
         int tfinal = 0;
+        int bfirst = INT_MAX, blast = -1;  // bottom row's first/last live column (from the parked values)
+        if constexpr (PIPE) lastlive = s == 0 ? -1 : INT_MAX;  // unknown until strip s-1 has finished
+
+        // park steps [st0, stmax] (at most 16) of lane 31's outputs in the ring (lanes 0..15); track live columns
+        auto park = [&](int st0, int stmax) {
+            const int st = st0 + lane, rc31 = st - 31;
+            const bool ok = lane < 16 && st <= stmax && rc31 >= 0 && rc31 <= span;
+            int xv = NEG;
+            if (ok) {
+                xv = ws->bout[0][st & 31];
+                ring[(start + rc31) & rmask] = make_int4(xv, ws->bout[1][st & 31], ws->bout[2][st & 31], 0);
+            }
+            const unsigned bal = __ballot_sync(FULL, ok && xv != NEG);
+            if (bal) {
+                const int c0 = start + st0 - 31;  // column of lane 0's entry
+                if (bfirst == INT_MAX) bfirst = c0 + __ffs(bal) - 1;
+                blast = c0 + 31 - __clz(bal);
+            }
+            if constexpr (PIPE) {
+                const unsigned okb = __ballot_sync(FULL, ok);
+                if (okb) {
+                    __threadfence_block();
+                    if (lane == 0) {
+                        const int c0 = start + st0 - 31;
+                        ps->first[slot] = bfirst;
+                        ps->last[slot] = blast;
+                        ps->prog[slot] = c0 + 31 - __clz(okb);
+                    }
+                }
+            }
+        };
 
         // one wavefront step: lane computes column start + tt - lane.  Returns true when the strip is done.
         auto step = [&](auto chk, auto eag, const int tt, const int u, const int j, const int cbase) -> bool {
@@ -244,9 +394,25 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                 // done at lane 31's column x = start + tt - 31 iff every lane has been dead since it processed
                 // x (step tt - 31 + lane) and the boundary row has no live cell at or after x
                 const unsigned bal = __ballot_sync(FULL, lastlive_t < tt - 31 + lane);
-                if (bal == FULL && start + tt - 31 > lastlive) {
-                    tfinal = tt;
-                    return true;
+                if (bal == FULL) {
+                    if constexpr (PIPE) {
+                        // deterministic (== SOLO): decide only once strip s-1 has either finished or flushed a
+                        // live bottom cell at or after x; never on the timing of its progress
+                        const int x = start + tt - 31;
+                        while (lastlive == INT_MAX) {
+                            if (ps->done[pslot] == s - 1) {
+                                __threadfence_block();
+                                lastlive = ps->last[pslot];
+                                break;
+                            }
+                            if (ps->last[pslot] >= x) break;  // not done at x; lastlive stays unknown
+                            pipe_wait();
+                        }
+                    }
+                    if (start + tt - 31 > lastlive) {
+                        tfinal = tt;
+                        return true;
+                    }
                 }
             }
             if (CHK && tt == tlast) {
@@ -260,19 +426,17 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         for (;;) {
             if (t > 0) {
                 __syncwarp();  // lane 31's parked rows of the previous block -> visible to lanes 0..15
-                // staging refills for relative columns [t+16, t+32), prefetch [t+32, t+48); park -> ring
+                park(t - 16, t - 1);
+                pipe_sync(start + t + 47);
+                // staging refills for relative columns [t+16, t+32), prefetch [t+32, t+48)
                 if (lane < 16) {
                     const int rcn = t + 16 + lane;
                     ws->bin[0][rcn & 31] = bpre.x;
                     ws->bin[1][rcn & 31] = bpre.y;
                     ws->bin[2][rcn & 31] = bpre.z;
                     cp_store(io, rcn, qpre);
-                    bpre = boundary(ring, rmask, start + rcn + 16, Emax, Wfar);
+                    bpre = boundary<PIPE>(ring, rmask, start + rcn + 16, blim, bwf);
                     qpre = query_code(io, start + rcn + 16);
-                    const int st = t - 16 + lane, rc31 = st - 31;
-                    if (rc31 >= 0 && rc31 <= span)
-                        ring[(start + rc31) & rmask] =
-                            make_int4(ws->bout[0][st & 31], ws->bout[1][st & 31], ws->bout[2][st & 31], 0);
                 }
             }
             __syncwarp();
@@ -306,66 +470,85 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         // ------------------------------------------------------------------ strip finish
         const int e = start + tfinal - 31;  // lane 31's last column
         __syncwarp();
-        if (lane < 16) {  // park the last (partial) block's bottom rows in the ring
-            const int st = t + lane, rc31 = st - 31;
-            if (st <= tfinal && rc31 >= 0 && rc31 <= span)
-                ring[(start + rc31) & rmask] =
-                    make_int4(ws->bout[0][st & 31], ws->bout[1][st & 31], ws->bout[2][st & 31], 0);
-        }
+        park(t, tfinal);  // the last (partial) block's bottom rows
         if constexpr (MODE == MODE_EXEC) {
             if ((tfinal % SPW) != SPW - 1) io.codes[wbase + (long long)(tfinal / SPW) * 32 + lane] = cw;
         }
-        cum_words += (long long)(tfinal / SPW + 1) * 32;
-        if constexpr (MODE == MODE_INSPECT) {
-            if (__any_sync(FULL, upd)) bound_words = cum_words;
-            upd = false;
-        }
         const int Wtail = ws->bout[2][tfinal & 31];
+        const int sw = (tfinal / SPW + 1) * 32;
+        const bool anyupd = __any_sync(FULL, upd);
+        upd = false;
+        if constexpr (PIPE) {  // the side state is sequential: wait for strip s-1's finish
+            if (s > 0) {
+                while (ps->done[pslot] != s - 1) pipe_wait();
+                __threadfence_block();
+            }
+            Emax = ps->Emax;
+            Wfar = ps->Wfar;
+            cum_words = ps->cum_words;
+            bound_words = ps->bound_words;
+            maxsw = ps->maxsw;
+            bound_maxsw = ps->bound_maxsw;
+            flags = ps->flags;
+        }
+        cum_words += sw;
+        maxsw = sw > maxsw ? sw : maxsw;
+        if (MODE == MODE_INSPECT && anyupd) {
+            bound_words = cum_words;
+            bound_maxsw = maxsw;
+        }
+        bool over = false;
         if (e - start + 4 > rmask) {  // strip wider than the ring: the parked row has been overwritten
             flags |= SF_RING;
-            break;
+            over = true;
         }
-        __syncwarp();
-        // V of the boundary row beyond e: max of the old boundary and this strip's tail (exact, reading R3)
-        for (int c = e + 1 + lane; c <= Emax; c += 32) {
-            const int4 v = ring[c & rmask];
-            ring[c & rmask] = make_int4(NEG, NEG, imax(v.z, Wtail), 0);
-        }
-        if (e >= Emax) {
-            Emax = e;
-            Wfar = Wtail;
-        } else {
-            Wfar = imax(Wfar, Wtail);
-        }
-        int first = INT_MAX, last = -1;
-        for (int c0 = start; c0 <= e; c0 += 32) {
-            const int c = c0 + lane;
-            const bool lv = c <= e && ring[c & rmask].x != NEG;
-            const unsigned bal = __ballot_sync(FULL, lv);
-            if (bal) {
-                if (first == INT_MAX) first = c0 + __ffs(bal) - 1;
-                last = c0 + 31 - __clz(bal);
+        if (!over) {
+            __syncwarp();
+            // V of the boundary row beyond e: max of the old boundary and this strip's tail (exact, reading R3)
+            for (int c = e + 1 + lane; c <= Emax; c += 32) {
+                const int4 v = PIPE ? __ldcg(ring + (c & rmask)) : ring[c & rmask];
+                ring[c & rmask] = make_int4(NEG, NEG, imax(v.z, Wtail), 0);
             }
-        }
-        __syncwarp();
-        if (MODE == MODE_INSPECT) {
-            // int32 range guard (reading R8)
-            if (__any_sync(FULL, best + OE >= SCORE_LIMIT)) {
+            if (e >= Emax) {
+                Emax = e;
+                Wfar = Wtail;
+            } else {
+                Wfar = imax(Wfar, Wtail);
+            }
+            if (MODE == MODE_INSPECT && __any_sync(FULL, best + OE >= SCORE_LIMIT)) {  // int32 guard (R8)
                 flags |= SF_OVERFLOW;
-                break;
+                over = true;
+            }
+            if (top + H > M || blast < 0) over = true;  // matrix bottom, or no live cell: extension ends (R6)
+            if (!over && Emax + 4 - bfirst > rmask) {   // boundary band wider than the ring
+                flags |= SF_RING;
+                over = true;
             }
         }
-        if (top + H > M || last < 0) break;  // matrix bottom reached, or no live cell: extension ends (R6)
-        if (Emax + 4 - first > rmask) {      // boundary band wider than the ring
-            flags |= SF_RING;
-            break;
-        }
-        if (first > start) Wleft0 = ring[(first - 1) & rmask].z;
-        lastlive = last;
-        start = first;
         __syncwarp();
+        if constexpr (PIPE) {
+            if (lane == 0) {
+                ps->Emax = Emax;
+                ps->Wfar = Wfar;
+                ps->cum_words = cum_words;
+                ps->bound_words = bound_words;
+                ps->maxsw = maxsw;
+                ps->bound_maxsw = bound_maxsw;
+                ps->flags = flags;
+                if (over) ps->end_strip = s;
+                __threadfence_block();
+                ps->done[slot] = s;
+            }
+            __syncwarp();
+            if (over) break;
+        } else {
+            if (over) break;
+            lastlive = blast;
+            nfirst = bfirst;
+            __syncwarp();
+        }
     }
-
+side_done:
     if constexpr (MODE == MODE_INSPECT) {
 #pragma unroll
         for (int off = 16; off; off >>= 1) {
@@ -379,6 +562,29 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             }
         }
     }
+    if constexpr (PIPE) {
+        if (lane == 0) {
+            ps->best[io.wi] = best;
+            ps->bi[io.wi] = bi;
+            ps->bj[io.wi] = bj;
+        }
+        __syncthreads();
+        best = ps->best[0];
+        bi = ps->bi[0];
+        bj = ps->bj[0];
+        for (int w = 1; w < io.K; ++w) {
+            const int ob = ps->best[w], oi = ps->bi[w], oj = ps->bj[w];
+            if (ob > best || (ob == best && (oi < bi || (oi == bi && oj < bj)))) {
+                best = ob;
+                bi = oi;
+                bj = oj;
+            }
+        }
+        flags = ps->flags;
+        bound_words = ps->bound_words;
+        bound_maxsw = ps->bound_maxsw;
+        cum_words = ps->cum_words;
+    }
     if constexpr (MODE == MODE_CENSUS) {
 #pragma unroll
         for (int off = 16; off; off >>= 1) cells += __shfl_xor_sync(FULL, cells, off);
@@ -388,8 +594,28 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
     out.bj = bj;
     out.flags = flags;
     out.bound_words = bound_words;
+    out.bound_maxsw = bound_maxsw;
     out.cells = cells;
     out.words = cum_words;
+}
+
+// Reset the block-per-problem shared state before a side (one thread; caller synchronises the CTA).
+__device__ __forceinline__ void pipe_reset(PipeShared* ps) {
+    for (int k = 0; k < PIPE_SLOTS; ++k) {
+        ps->sid[k] = -1;
+        ps->done[k] = -1;
+        ps->first[k] = INT_MAX;
+        ps->last[k] = -1;
+        ps->prog[k] = -1;
+    }
+    ps->end_strip = INT_MAX;
+    ps->Emax = -1;
+    ps->Wfar = NEG;
+    ps->flags = 0;
+    ps->cum_words = 0;
+    ps->bound_words = 0;
+    ps->maxsw = 0;
+    ps->bound_maxsw = 0;
 }
 
 }  // namespace fz

@@ -155,3 +155,40 @@ def test_unfolded_profile_large_scores():
     bad, *_ = compare(T, Q, seeds, sub=hox * 200, gap_open=8000, gap_extend=600, ydrop=8000 + 300 * 600,
                       gapped_threshold=600000)
     assert_ok(bad)
+
+
+@pytest.fixture
+def force_block(monkeypatch):
+    """Every side that needs more than one strip escalates to the block-per-side inspector and every executed
+    side runs block per side (pipelined strips across the CTA's warps)."""
+    monkeypatch.setenv("FASTZ_ESCALATE_STRIPS", "1")
+    monkeypatch.setenv("FASTZ_BLOCK_BIN", "1")
+
+
+def test_block_per_side_mixed(force_block):
+    for seed in range(2):
+        w = genome.small_pair(40 + seed, length=20000, n_seeds=200)
+        bad, *_ = compare(w.T, w.Q, w.seeds, census=False)
+        assert_ok(bad)
+
+
+def test_block_per_side_long_and_adversarial(force_block):
+    rng = random.Random(19)
+    T = rseq(rng, 9000)
+    Q = mutate(rng, T, sub=0.08, indel=0.01)
+    seeds = [(4500, int(len(Q) * 0.5)), (0, 0), (9000, len(Q)), (100, 90)]
+    bad, *_ = compare(T, Q, seeds, census=False)
+    assert_ok(bad)
+    for Y in (0, 300, 10 ** 6):
+        bad, *_ = compare(T[:3000], Q[:3000], [(1500, 1500), (0, 0), (3000, 3000)], census=False, ydrop=Y)
+        assert_ok(bad)
+    bad, *_ = compare("A" * 3000, "A" * 2500, [(0, 0), (1000, 1000), (3000, 2500)], census=False)
+    assert_ok(bad)
+
+
+def test_block_inspector_only(monkeypatch):
+    """Escalation after 2 strips with the default executor split."""
+    monkeypatch.setenv("FASTZ_ESCALATE_STRIPS", "2")
+    w = genome.small_pair(50, length=30000, n_seeds=150)
+    bad, *_ = compare(w.T, w.Q, w.seeds, census=False)
+    assert_ok(bad)
