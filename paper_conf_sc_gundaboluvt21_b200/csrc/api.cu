@@ -12,6 +12,7 @@
 #include <cstdio>
 #include <cstring>
 #include <string>
+#include <vector>
 
 #include "../../include/fastz.h"
 #include "internal.h"
@@ -51,10 +52,11 @@ struct fastz_ctx {
     int tlen = 0, qlen = 0;
     DBuf Tf, Tr, Qf, Qr, stage;
     DBuf seeds, score, ti, qj, flags, eops, bound, maxsw, esc;
-    DBuf woff, soff, roff, bin, list, counters, totals, tmpa, tmpb, tmpc, scan_tmp;
+    DBuf woff, soff, roff, bin, list, counters, totals, tmpa, tmpb, tmpc, scan_tmp, wl, wlo;
     DBuf codes, stab, runs, nruns, ciglen, cigar, recs, cells, ring, small;
     int R = 4, grid = 0, nslots = 0, rmask = 0;
     int64_t n = 0, cigar_bytes = 0, nexec = 0;
+    int nwaves = 0;
     bool have = false;
     fastz_stats stats{};
     cudaEvent_t ev[8] = {};
@@ -196,6 +198,8 @@ ExecPlan make_plan(fastz_ctx* c) {
     p.counters = P_<int>(c->counters);
     p.totals = P_<long long>(c->totals);
     p.esc = P_<int>(c->esc);
+    p.wl = P_<long long>(c->wl);
+    p.wlo = P_<long long>(c->wlo);
     return p;
 }
 
@@ -259,7 +263,7 @@ void fastz_destroy(fastz_ctx* c) {
     if (c->stream) cudaStreamSynchronize(c->stream);
     DBuf* bufs[] = {&c->Tf, &c->Tr, &c->Qf, &c->Qr, &c->stage, &c->seeds, &c->score, &c->ti, &c->qj,
                     &c->flags, &c->eops, &c->bound, &c->maxsw, &c->esc, &c->woff, &c->soff, &c->roff, &c->bin, &c->list,
-                    &c->counters, &c->totals, &c->tmpa, &c->tmpb, &c->tmpc, &c->scan_tmp, &c->codes,
+                    &c->counters, &c->totals, &c->tmpa, &c->tmpb, &c->tmpc, &c->scan_tmp, &c->wl, &c->wlo, &c->codes,
                     &c->stab, &c->runs, &c->nruns, &c->ciglen, &c->cigar, &c->recs, &c->cells, &c->ring,
                     &c->small};
     for (DBuf* b : bufs) dfree(c, *b);
@@ -363,6 +367,8 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     AL(tmpa, std::max<int64_t>(ns, 1) * 8);
     AL(tmpb, std::max<int64_t>(ns, 1) * 8);
     AL(tmpc, std::max<int64_t>(ns, 1) * 8);
+    AL(wl, std::max<int64_t>(ns, 1) * 8);
+    AL(wlo, std::max<int64_t>(ns, 1) * 8);
     AL(nruns, std::max<int64_t>(ns, 1) * 4);
     AL(ciglen, std::max<int64_t>(2 * n, 1) * 8);
     AL(recs, std::max<int64_t>(n, 1) * sizeof(fastz_alignment));
@@ -408,15 +414,56 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     const long long words = h.totals[0], strips = h.totals[1], nrun = h.totals[2];
     c->nexec = h.totals[3];
     const long long nblock = h.totals[4];
-    AL(codes, std::max<long long>(words, 1) * 4);
     AL(stab, std::max<long long>(strips, 1) * 8);
     AL(runs, std::max<long long>(nrun, 1) * 4);
+    // traceback-code pool: one wave if it fits the budget, else consecutive ranges of the executor list
+    // (largest bins first), each executed and traced back before the pool is reused
+    long long budget_words;
+    {
+        const char* e = getenv("FASTZ_POOL_MB");
+        if (e) {
+            budget_words = std::max<long long>(atoll(e), 1) * (1LL << 20) / 4;
+        } else {
+            size_t fr = 0, tot = 0;
+            cudaMemGetInfo(&fr, &tot);
+            budget_words = (long long)((fr + c->codes.cap) / 2 / 4);
+        }
+    }
+    std::vector<std::pair<long long, long long>> waves;  // list ranges [a, b)
+    std::vector<long long> wbase;
+    long long pool_words = words;
+    if (words <= budget_words || c->nexec <= 1) {
+        waves.push_back({0, c->nexec});
+        wbase.push_back(0);
+    } else {
+        std::vector<long long> wlo((size_t)c->nexec + 1);
+        CK(cudaMemcpyAsync(wlo.data(), c->wlo.p, (size_t)c->nexec * 8, cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        wlo[(size_t)c->nexec] = words;
+        pool_words = 0;
+        long long a = 0;
+        while (a < c->nexec) {
+            long long b = a + 1;
+            while (b < c->nexec && wlo[(size_t)b + 1] - wlo[(size_t)a] <= budget_words) ++b;
+            waves.push_back({a, b});
+            wbase.push_back(wlo[(size_t)a]);
+            pool_words = std::max(pool_words, wlo[(size_t)b] - wlo[(size_t)a]);
+            a = b;
+        }
+    }
+    AL(codes, std::max<long long>(pool_words, 1) * 4);
     Outputs o = make_out(c);
-    CK(launch_execute(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, (int)c->nexec, (int)nblock, o,
-                      st));
-    CK(cudaEventRecord(c->ev[4], st));
-    CK(launch_traceback(c->R, sa, pl, (int)c->nexec, o, st));
+    for (size_t w = 0; w < waves.size(); ++w) {
+        if (w) CK(cudaMemsetAsync(P_<int>(c->counters) + 1, 0, 4, st));
+        if (w) CK(cudaMemsetAsync(P_<int>(c->counters) + 23, 0, 4, st));
+        CK(launch_execute(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, (int)waves[w].first,
+                          (int)waves[w].second, (int)nblock, wbase[w], o, st));
+        if (w == 0) CK(cudaEventRecord(c->ev[4], st));
+        CK(launch_traceback(c->R, sa, pl, (int)waves[w].first, (int)waves[w].second, wbase[w], o, st));
+    }
+    if (waves.empty()) CK(cudaEventRecord(c->ev[4], st));
     CK(cudaEventRecord(c->ev[5], st));
+    c->nwaves = (int)waves.size();
     long long* dtotal = P_<long long>(c->small) + 1;
     CK(launch_combine_len(c->dp, b, sa, pl, o, c->scan_tmp.p, stb, dtotal, st));
     long long ctot = 0;

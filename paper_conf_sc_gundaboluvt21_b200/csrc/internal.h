@@ -39,6 +39,8 @@ struct ExecPlan {
                          // [23] executor block queue
     long long* totals;   // [0] words, [1] strips, [2] runs, [3] n_exec, [4] n_exec_block
     int* esc;            // escalated sides (inspector -> block inspector)
+    long long* wl;       // executor words in list order (scratch)
+    long long* wlo;      // exclusive scan of wl: pool offset of list position i
 };
 
 struct Outputs {
@@ -70,10 +72,11 @@ cudaError_t launch_bin(int R, const SideArrays& sa, int nsides, const ExecPlan& 
                        cudaStream_t st);
 size_t scan_tmp_bytes(int n);
 cudaError_t launch_execute(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
-                           const SideArrays& sa, const ExecPlan& pl, int nexec, int nblock, const Outputs& o,
+                           const SideArrays& sa, const ExecPlan& pl, int lo, int hi, int nblock, long long base,
+                           const Outputs& o,
                            cudaStream_t st);
-cudaError_t launch_traceback(int R, const SideArrays& sa, const ExecPlan& pl, int nexec, const Outputs& o,
-                             cudaStream_t st);
+cudaError_t launch_traceback(int R, const SideArrays& sa, const ExecPlan& pl, int lo, int hi, long long base,
+                             const Outputs& o, cudaStream_t st);
 cudaError_t launch_combine_len(const DevParams& P, const Batch& b, const SideArrays& sa, const ExecPlan& pl,
                                const Outputs& o, void* scan_tmp, size_t scan_tmp_bytes, long long* total,
                                cudaStream_t st);

@@ -252,8 +252,8 @@ __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int
 // across the CTA's warps), then every warp takes short sides (bins 1-2, warp per side), larger bins first.
 template <int R, bool FOLD>
 __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, int4* ring, int rmask,
-                                                         SideArrays sa, ExecPlan pl, int nexec, int nblock,
-                                                         Outputs out) {
+                                                         SideArrays sa, ExecPlan pl, int lo, int hi, int nblock,
+                                                         long long base, Outputs out) {
     __shared__ SmemDP sm;
     __shared__ PipeShared ps;
     __shared__ int cur;
@@ -261,8 +261,8 @@ __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, in
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     for (;;) {  // block phase
         if (threadIdx.x == 0) {
-            const int i = atomicAdd(&pl.counters[23], 1);
-            cur = i < nblock ? pl.list[i] : -1;
+            const int i = lo + atomicAdd(&pl.counters[23], 1);
+            cur = i < (hi < nblock ? hi : nblock) ? pl.list[i] : -1;
             pipe_reset(&ps);
         }
         __syncthreads();
@@ -274,7 +274,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, in
         setup_side(b, side, io);
         io.M = sa.ti[side];
         io.N = sa.qj[side];
-        io.codes = out.codes + pl.woff[side];
+        io.codes = out.codes + (pl.woff[side] - base);
         io.stab = out.stab + pl.soff[side];
         io.maxsw = sa.maxsw[side];
         SideOut o;
@@ -286,14 +286,14 @@ __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, in
     io_init(io, sm, ring, rmask, blockIdx.x * WARPS + warp, warp);
     for (;;) {  // warp phase
         int idx = 0;
-        if (lane == 0) idx = nblock + atomicAdd(&pl.counters[1], 1);
+        if (lane == 0) idx = (lo > nblock ? lo : nblock) + atomicAdd(&pl.counters[1], 1);
         idx = __shfl_sync(FULL, idx, 0);
-        if (idx >= nexec) break;
+        if (idx >= hi) break;
         const int side = pl.list[idx];
         setup_side(b, side, io);
         io.M = sa.ti[side];
         io.N = sa.qj[side];
-        io.codes = out.codes + pl.woff[side];
+        io.codes = out.codes + (pl.woff[side] - base);
         io.stab = out.stab + pl.soff[side];
         SideOut o;
         run_side<R, MODE_EXEC, false, FOLD, false>(P, io, o);
@@ -306,12 +306,12 @@ __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, in
 // One thread per executed side (inter-seed traceback parallelism).  Walks the 4-bit codes from
 // (i*, j*) in state S to the origin; emits run-length ops (len << 2 | op) in peak -> origin order.
 template <int R>
-__global__ void k_traceback(SideArrays sa, ExecPlan pl, int nexec, Outputs out) {
+__global__ void k_traceback(SideArrays sa, ExecPlan pl, int lo, int hi, long long base, Outputs out) {
     constexpr int H = 32 * R, SPW = 8 / R;
-    const int idx = blockIdx.x * blockDim.x + threadIdx.x;
-    if (idx >= nexec) return;
+    const int idx = lo + blockIdx.x * blockDim.x + threadIdx.x;
+    if (idx >= hi) return;
     const int side = pl.list[idx];
-    const uint32_t* __restrict__ codes = out.codes + pl.woff[side];
+    const uint32_t* __restrict__ codes = out.codes + (pl.woff[side] - base);
     const int2* __restrict__ stab = out.stab + pl.soff[side];
     uint32_t* __restrict__ runs = out.runs + pl.roff[side];
     int i = sa.ti[side], j = sa.qj[side], state = 0, nr = 0;
@@ -394,7 +394,6 @@ __global__ void k_bin_offsets(ExecPlan pl, int nsides, const long long* words, c
         if (bin == bblock) nblock = run;
     }
     if (nsides > 0) {
-        pl.totals[0] = pl.woff[nsides - 1] + words[nsides - 1];
         pl.totals[1] = pl.soff[nsides - 1] + strips[nsides - 1];
         pl.totals[2] = pl.roff[nsides - 1] + runs[nsides - 1];
     } else {
@@ -402,6 +401,18 @@ __global__ void k_bin_offsets(ExecPlan pl, int nsides, const long long* words, c
     }
     pl.totals[3] = run;
     pl.totals[4] = nblock;
+}
+
+// pool offsets in executor (list) order, so that a wave is a contiguous range of the list
+__global__ void k_list_words(ExecPlan pl, const long long* words, long long* wl) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < (int)pl.totals[3]) wl[i] = words[pl.list[i]];
+}
+__global__ void k_list_offsets(ExecPlan pl, const long long* wlo, const long long* wl) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    const int n = (int)pl.totals[3];
+    if (i < n) pl.woff[pl.list[i]] = wlo[i];
+    if (i == 0) pl.totals[0] = n > 0 ? wlo[n - 1] + wl[n - 1] : 0;
 }
 
 __global__ void k_bin_scatter(ExecPlan pl, int nsides) {
@@ -428,22 +439,27 @@ size_t scan_tmp_bytes(int n) {
 cudaError_t launch_bin(int R, const SideArrays& sa, int nsides, const ExecPlan& pl, void* tmp, size_t tmp_bytes,
                        long long* words, long long* strips, long long* runs, cudaStream_t st) {
     const int bb = block_bin();
+    cudaError_t e;
     if (nsides > 0) {
         const int g = (nsides + 255) / 256;
-        switch (R) {
-            case 2: k_bin_count<2><<<g, 256, 0, st>>>(sa, nsides, pl, words, strips, runs, bb); break;
-            default: k_bin_count<4><<<g, 256, 0, st>>>(sa, nsides, pl, words, strips, runs, bb); break;
-        }
-        cudaError_t e;
+        if (R == 2) k_bin_count<2><<<g, 256, 0, st>>>(sa, nsides, pl, words, strips, runs, bb);
+        else k_bin_count<4><<<g, 256, 0, st>>>(sa, nsides, pl, words, strips, runs, bb);
         size_t b = tmp_bytes;
-        if ((e = cub::DeviceScan::ExclusiveSum(tmp, b, words, pl.woff, nsides, st)) != cudaSuccess) return e;
-        b = tmp_bytes;
         if ((e = cub::DeviceScan::ExclusiveSum(tmp, b, strips, pl.soff, nsides, st)) != cudaSuccess) return e;
         b = tmp_bytes;
         if ((e = cub::DeviceScan::ExclusiveSum(tmp, b, runs, pl.roff, nsides, st)) != cudaSuccess) return e;
     }
     k_bin_offsets<<<1, 1, 0, st>>>(pl, nsides, words, strips, runs, bb);
-    if (nsides > 0) k_bin_scatter<<<(nsides + 255) / 256, 256, 0, st>>>(pl, nsides);
+    if (nsides > 0) {
+        const int g = (nsides + 255) / 256;
+        k_bin_scatter<<<g, 256, 0, st>>>(pl, nsides);
+        long long* wl = pl.wl;
+        long long* wlo = pl.wlo;
+        k_list_words<<<g, 256, 0, st>>>(pl, words, wl);
+        size_t b = tmp_bytes;
+        if ((e = cub::DeviceScan::ExclusiveSum(tmp, b, wl, wlo, nsides, st)) != cudaSuccess) return e;
+        k_list_offsets<<<g, 256, 0, st>>>(pl, wlo, wl);
+    }
     return cudaGetLastError();
 }
 
@@ -632,21 +648,19 @@ cudaError_t launch_census(int R, int grid, const DevParams& P, const Batch& b, i
 }
 
 cudaError_t launch_execute(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
-                           const SideArrays& sa, const ExecPlan& pl, int nexec, int nblock, const Outputs& o,
-                           cudaStream_t st) {
-    if (nexec == 0) return cudaSuccess;
-    FZ_DISPATCH(k_execute, grid, P, b, ring, rmask, sa, pl, nexec, nblock, o);
+                           const SideArrays& sa, const ExecPlan& pl, int lo, int hi, int nblock, long long base,
+                           const Outputs& o, cudaStream_t st) {
+    if (hi <= lo) return cudaSuccess;
+    FZ_DISPATCH(k_execute, grid, P, b, ring, rmask, sa, pl, lo, hi, nblock, base, o);
     return cudaGetLastError();
 }
 
-cudaError_t launch_traceback(int R, const SideArrays& sa, const ExecPlan& pl, int nexec, const Outputs& o,
-                             cudaStream_t st) {
-    if (nexec == 0) return cudaSuccess;
-    const int g = (nexec + 127) / 128;
-    switch (R) {
-        case 2: k_traceback<2><<<g, 128, 0, st>>>(sa, pl, nexec, o); break;
-        default: k_traceback<4><<<g, 128, 0, st>>>(sa, pl, nexec, o); break;
-    }
+cudaError_t launch_traceback(int R, const SideArrays& sa, const ExecPlan& pl, int lo, int hi, long long base,
+                             const Outputs& o, cudaStream_t st) {
+    if (hi <= lo) return cudaSuccess;
+    const int g = (hi - lo + 127) / 128;
+    if (R == 2) k_traceback<2><<<g, 128, 0, st>>>(sa, pl, lo, hi, base, o);
+    else k_traceback<4><<<g, 128, 0, st>>>(sa, pl, lo, hi, base, o);
     return cudaGetLastError();
 }
 

@@ -192,3 +192,16 @@ def test_block_inspector_only(monkeypatch):
     w = genome.small_pair(50, length=30000, n_seeds=150)
     bad, *_ = compare(w.T, w.Q, w.seeds, census=False)
     assert_ok(bad)
+
+
+def test_executor_waves_under_pool_budget(monkeypatch):
+    """A 1 MiB traceback-code budget forces the executor + traceback into many waves (list ranges)."""
+    monkeypatch.setenv("FASTZ_POOL_MB", "1")
+    w = genome.small_pair(60, length=30000, n_seeds=200)
+    bad, *_ = compare(w.T, w.Q, w.seeds, census=False)
+    assert_ok(bad)
+    rng = random.Random(61)
+    T = rseq(rng, 6000)
+    Q = mutate(rng, T, sub=0.08, indel=0.01)
+    bad, *_ = compare(T, Q, [(3000, int(len(Q) * 0.5)), (0, 0), (6000, len(Q)), (10, 10)], census=False)
+    assert_ok(bad)
