@@ -203,6 +203,7 @@ def run_fastz(args, ws, rank, local):
         dist.barrier()
     clk = Clocks(local)
     times, insp, stages = [], [], []
+    launches = 0
     for _ in range(args.steps):
         flush.zero_()  # L2 flushed between timed steps (outside the events)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -215,6 +216,7 @@ def run_fastz(args, ws, rank, local):
         s = al.stats()
         insp.append(s["ms_inspect"])
         stages.append(s)
+        launches += int(s["n_launches"])
     torch.cuda.synchronize()
     clocks = clk.stop()
     if ws > 1:
@@ -235,6 +237,14 @@ def run_fastz(args, ws, rank, local):
         e2e_t.append(time.perf_counter() - t0)
         d2h = res.rec.nbytes + len(res.cigar)
     e2e_ms = sum(e2e_t) / len(e2e_t) * 1e3
+
+    # genome-pair wall time: ASCII sequences + seeds on the host -> alignments + CIGARs on the host
+    # (context creation with device packing, extension, copy-back), seed finding excluded
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    with fastz.Aligner(w.T, w.Q, device=local, stream=stream.cuda_stream) as al2:
+        al2.extend(np.ascontiguousarray(shard))
+    wall_s = time.perf_counter() - t0
 
     t = torch.tensor([ms, e2e_ms, float(cells), float(n)], dtype=torch.float64, device=dev)
     if ws > 1:
@@ -271,7 +281,8 @@ def run_fastz(args, ws, rank, local):
         "clocks": clocks,
         "e2e": {"value": cells_all / (e2e_ms * 1e-3) / 1e9, "unit": "GCUPS", "ms_per_step": e2e_ms,
                 "h2d_bytes_per_step": int(n * 16), "d2h_bytes_per_step": int(d2h)},
-        "gpu_launches": 10 * args.steps,
+        "gpu_launches": launches,
+        "genome_pair_wall_s": wall_s,
         "roofline": {"bound": "alu", "kernel": "k_inspect", "achieved": achieved / 1e12, "peak": peak_ops / 1e12,
                      "unit": "Tops/s (INT32 lane ops)", "frac": achieved / peak_ops, "traffic": traffic,
                      "ops_per_cell": OPS_PER_CELL, "inspector_ms": insp_ms,
@@ -279,6 +290,7 @@ def run_fastz(args, ws, rank, local):
         "stages_ms": {k: avg(k) for k in ("ms_upload", "ms_inspect", "ms_bin", "ms_execute", "ms_traceback",
                                           "ms_combine")},
         "bins_per_side": st0["bin_counts"][:7], "exec_sides": st0["n_exec_sides"], "eager_sides": st0["n_eager_sides"],
+        "escalated_sides": st0["n_escalated"], "executor_waves": st0["n_waves"],
     }
     if not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(w, shard)

@@ -157,6 +157,9 @@ typedef struct {
                                      5 <=131072, 6 larger (4x rule) */
     int64_t exec_words;           /* 32-bit traceback-code words written by the executor */
     int64_t cigar_bytes;
+    int64_t n_launches;           /* kernels of this library launched by the call (CUB scans excluded) */
+    int64_t n_waves;              /* executor/traceback waves under the traceback-pool budget */
+    int64_t n_escalated;          /* sides handed from the warp inspector to the block inspector */
 } fastz_stats;
 int fastz_get_stats(fastz_ctx *c, fastz_stats *s);
 

@@ -485,6 +485,11 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     for (int k = 0; k < 7; ++k) S.bin_counts[k] = h.counters[2 + k];
     S.exec_words = words;
     S.cigar_bytes = ctot;
+    S.n_waves = c->nwaves;
+    S.n_escalated = h.counters[21];
+    // own kernels: validate, inspect, inspect_block (if escalation on), bin_count, bin_offsets, bin_scatter,
+    // list_words, list_offsets, execute + traceback per wave, combine_len, combine_total, combine_write
+    S.n_launches = (n > 0 ? 1 + 1 + (esc > 0 ? 1 : 0) + 5 + 2 * (int64_t)c->nwaves + 3 : 1);
     c->have = true;
     return 0;
 }

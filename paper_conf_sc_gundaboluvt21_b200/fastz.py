@@ -45,7 +45,8 @@ class fastz_stats(ctypes.Structure):
                 ("ms_bin", ctypes.c_float), ("ms_execute", ctypes.c_float), ("ms_traceback", ctypes.c_float),
                 ("ms_combine", ctypes.c_float), ("n_warp_slots", ctypes.c_int32), ("n_seeds", ctypes.c_int64),
                 ("n_sides", ctypes.c_int64), ("n_eager_sides", ctypes.c_int64), ("n_exec_sides", ctypes.c_int64),
-                ("bin_counts", ctypes.c_int64 * 8), ("exec_words", ctypes.c_int64), ("cigar_bytes", ctypes.c_int64)]
+                ("bin_counts", ctypes.c_int64 * 8), ("exec_words", ctypes.c_int64), ("cigar_bytes", ctypes.c_int64),
+                ("n_launches", ctypes.c_int64), ("n_waves", ctypes.c_int64), ("n_escalated", ctypes.c_int64)]
 
 
 ALIGN_DTYPE = np.dtype([("score", "<i4"), ("left_score", "<i4"), ("right_score", "<i4"), ("flags", "<u4"),

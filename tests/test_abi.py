@@ -72,12 +72,15 @@ def test_strerror_and_destroy_null():
     L.fastz_destroy(None)
 
 
-def test_sass_has_no_cpu_fallback_and_targets_sm100a():
-    """The library contains sm_100a SASS for the DP kernels (cuobjdump lists them)."""
-    out = subprocess.check_output(["/usr/local/cuda/bin/cuobjdump", "-lelf", build.build()]).decode()
-    assert "sm_100a" in out
-    sym = subprocess.check_output(["/usr/local/cuda/bin/cuobjdump", "-sass", "-fun",
-                                   "_ZN2fz9k_inspectILi4EEEvNS_9DevParamsENS_5BatchEP4int4iNS_10SideArraysEPi",
-                                   build.build()]).decode()
-    for mnem in ("VIADDMNMX", "VIMNMX3", "PRMT", "SHFL.UP", "VOTE"):
-        assert mnem in sym, mnem
+def test_sass_targets_sm100a_and_uses_the_integer_dp_instructions():
+    """The library contains sm_100a SASS for every DP kernel (inspector, block inspector, executor, census),
+    built from the fused integer instructions the design relies on."""
+    out = subprocess.check_output(["/usr/local/cuda/bin/cuobjdump", "-sass", build.build()]).decode()
+    sections = out.split("Function : ")
+    names = [sec.split("\n", 1)[0] for sec in sections[1:]]
+    for k in ("k_inspectILi4ELb1E", "k_inspect_blockILi4ELb1E", "k_executeILi4ELb1E", "k_censusILi4ELb1E",
+              "k_traceback", "k_pack", "k_bin_count", "k_combine_write"):
+        assert any(k in n for n in names), k
+    insp = next(sec for sec in sections[1:] if sec.startswith("_ZN2fz9k_inspectILi4ELb1E"))
+    for mnem in ("VIADDMNMX", "VIMNMX3", "PRMT", "SHFL.IDX", "VOTE", "IMAD"):
+        assert mnem in insp, mnem
