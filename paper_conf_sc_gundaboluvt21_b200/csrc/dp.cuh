@@ -70,6 +70,17 @@ __device__ __forceinline__ void ld_shared_if(bool p, unsigned addr, int& v) {
     asm volatile("{ .reg .pred q; setp.ne.u32 q, %1, 0; @q ld.shared.b32 %0, [%2]; }" : "+r"(v) : "r"((unsigned)p), "r"(addr));
 }
 
+// predicated 128-bit shared store / load of a register quad (x, y, z, w)
+__device__ __forceinline__ void st_shared4_if(bool p, unsigned addr, int4 v) {
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %0, 0; @q st.shared.v4.b32 [%1], {%2, %3, %4, %5}; }" ::"r"((unsigned)p),
+                 "r"(addr), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w));
+}
+__device__ __forceinline__ void ld_shared4_if(bool p, unsigned addr, int4& v) {
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %4, 0; @q ld.shared.v4.b32 {%0, %1, %2, %3}, [%5]; }"
+                 : "+r"(v.x), "+r"(v.y), "+r"(v.z), "+r"(v.w)
+                 : "r"((unsigned)p), "r"(addr));
+}
+
 __device__ __forceinline__ int prmt(int a, int b, int s) {
     int d;
     asm("prmt.b32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(s));

@@ -43,8 +43,9 @@ constexpr int PIPE_SLOTS = 8;  // 2K slots for K = 4 warps: a slot is reused onl
 
 struct WarpSmem {
     int2 cp[CP_RING + 16];  // column profiles, ring over relative columns (+16 mirrored)
-    int bin[3][32];         // boundary row staging (X, D, W; lane 0's input, served through lane 31)
-    int bout[3][32];        // lane 31's bottom-row outputs (X, D, W) awaiting the global ring
+    int4 bin[33];           // boundary row staging {X, D, W, -} (lane 0's input, served through lane 31);
+                            // entry 32 mirrors entry 0 so a 4-step group never wraps
+    int4 bout[32];          // lane 31's bottom-row outputs {X, D, W, -} awaiting the global ring
 };
 
 // Block-per-problem (PIPE) shared state of one side.  Strip s owns slot s % PIPE_SLOTS.
@@ -136,8 +137,8 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
     WarpSmem* __restrict__ ws = io.ws;
     PipeShared* __restrict__ ps = io.ps;
     const bool is31 = lane == 31;
-    const unsigned sb_in = (unsigned)__cvta_generic_to_shared(&ws->bin[0][0]);
-    const unsigned sb_out = (unsigned)__cvta_generic_to_shared(&ws->bout[0][0]);
+    const unsigned sb_in = (unsigned)__cvta_generic_to_shared(&ws->bin[0]);
+    const unsigned sb_out = (unsigned)__cvta_generic_to_shared(&ws->bout[0]);
 
     // W left of column 0 is V(i,-1) - Y = -inf; any value <= -Y gives the same thresholds (only the origin has
     // no finite neighbour, and it is live for any threshold <= 0).  -(Y+1) keeps the cells that lanes compute
@@ -213,7 +214,7 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             W[k] = (r <= M) ? Wleft0 : BIG;
         }
         int xdiag = (top == 0 && lane == 0) ? -OE : NEG;  // origin: H(0,0) = -OE + 0 + OE = 0
-        int xb = NEG, db = NEG, wb = NEG;
+        int4 bq = make_int4(NEG, NEG, NEG, 0);  // this lane's bottom row (X, D, W) -> lane + 1 (lane 31: boundary)
         const int span = N - start;
         const int tlast = span + 31;
         const long long wbase = PIPE ? (long long)s * io.maxsw : cum_words;  // executor: strip's first word
@@ -255,9 +256,8 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         // staging: boundary for relative columns [0, 32), column profiles [0, 32); prefetch the next 16
         {
             const int4 v = boundary<PIPE>(ring, rmask, start + lane, blim, bwf);
-            ws->bin[0][lane] = v.x;
-            ws->bin[1][lane] = v.y;
-            ws->bin[2][lane] = v.z;
+            ws->bin[lane] = v;
+            if (lane == 0) ws->bin[32] = v;
         }
         cp_store(io, lane, query_code(io, start + lane));
         int4 bpre = make_int4(NEG, NEG, bwf, 0);
@@ -267,13 +267,10 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             qpre = query_code(io, start + 32 + lane);
         }
         __syncwarp();
-        if (lane == 31) {
-            xb = ws->bin[0][0];
-            db = ws->bin[1][0];
-            wb = ws->bin[2][0];
-        }
+        if (lane == 31) bq = ws->bin[0];
         uint32_t cw = 0;
-        int lastlive_t = -1;  // last step at which this lane had a live cell (termination, see header)
+        int lastlive_t = -1;  // last 4-step group end at which this lane had a live cell (termination)
+        int cacc = NEG;       // max X of this lane over the current 4-step group
         int tfinal = 0;
         int bfirst = INT_MAX, blast = -1;  // bottom row's first/last live column (from the parked values)
         if constexpr (PIPE) lastlive = s == 0 ? -1 : INT_MAX;  // unknown until strip s-1 has finished
@@ -284,8 +281,9 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             const bool ok = lane < 16 && st <= stmax && rc31 >= 0 && rc31 <= span;
             int xv = NEG;
             if (ok) {
-                xv = ws->bout[0][st & 31];
-                ring[(start + rc31) & rmask] = make_int4(xv, ws->bout[1][st & 31], ws->bout[2][st & 31], 0);
+                const int4 v = ws->bout[st & 31];
+                xv = v.x;
+                ring[(start + rc31) & rmask] = v;
             }
             const unsigned bal = __ballot_sync(FULL, ok && xv != NEG);
             if (bal) {
@@ -308,14 +306,15 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         };
 
         // one wavefront step: lane computes column start + tt - lane.  Returns true when the strip is done.
-        auto step = [&](auto chk, auto eag, const int tt, const int u, const int j, const int cbase) -> bool {
+        auto step = [&](auto chk, auto eag, const int tt, const int u, const int j, const int cbase,
+                        const unsigned sgo, const unsigned sgi) -> bool {
             constexpr bool CHK = decltype(chk)::value;
             constexpr bool EG = decltype(eag)::value;
             const int rc = tt - lane;
             const bool valid = CHK ? (unsigned)rc <= (unsigned)span : true;
-            int xu = __shfl_sync(FULL, xb, src);
-            int du = __shfl_sync(FULL, db, src);
-            int wu = __shfl_sync(FULL, wb, src);
+            int xu = __shfl_sync(FULL, bq.x, src);
+            int du = __shfl_sync(FULL, bq.y, src);
+            int wu = __shfl_sync(FULL, bq.z, src);
             int cmv = NEG;
             if (valid) {
                 const int2 cp = ws->cp[cbase + u];
@@ -353,11 +352,10 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                     wu = wn;
                     cm = k == 0 ? xn : imax(cm, xn);
                 }
-                xb = xu;
-                db = du;
-                wb = wu;
-                // live -> tt, dead (cm == NEG) -> -1: one VIADDMNMX (min) + one max
-                lastlive_t = imax(lastlive_t, __viaddmin_s32(cm, -NEG - 1, tt));
+                bq.x = xu;
+                bq.y = du;
+                bq.z = wu;
+                cacc = imax(cacc, cm);
                 cmv = cm;
             }
             if constexpr (MODE == MODE_INSPECT) {
@@ -375,20 +373,19 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                     }
                 }
             }
-            {
-                const unsigned o = (unsigned)(tt & 31) * 4u, n = (unsigned)((tt + 1) & 31) * 4u;
-                st_shared_if(is31, sb_out + o, xb);
-                st_shared_if(is31, sb_out + 128u + o, db);
-                st_shared_if(is31, sb_out + 256u + o, wb);
-                ld_shared_if(is31, sb_in + n, xb);
-                ld_shared_if(is31, sb_in + 128u + n, db);
-                ld_shared_if(is31, sb_in + 256u + n, wb);
-            }
+            // lane 31 parks its bottom row and picks up the boundary for lane 0's next column
+            st_shared4_if(is31, sgo + 16u * (unsigned)j, bq);
+            ld_shared4_if(is31, sgi + 16u * (unsigned)j, bq);
             if constexpr (MODE == MODE_EXEC) {
                 if ((j % SPW) == SPW - 1) {  // j == tt mod 4 and SPW divides 4
                     io.codes[wbase + (long long)(tt / SPW) * 32 + lane] = cw;
                     cw = 0;
                 }
+            }
+            if (j == 3) {
+                // liveness per 4-step group: live anywhere in the group -> the group's last step (conservative)
+                lastlive_t = imax(lastlive_t, __viaddmin_s32(cacc, -NEG - 1, tt));
+                cacc = NEG;
             }
             if (j == 3 && tt >= 31) {
                 // done at lane 31's column x = start + tt - 31 iff every lane has been dead since it processed
@@ -431,9 +428,8 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                 // staging refills for relative columns [t+16, t+32), prefetch [t+32, t+48)
                 if (lane < 16) {
                     const int rcn = t + 16 + lane;
-                    ws->bin[0][rcn & 31] = bpre.x;
-                    ws->bin[1][rcn & 31] = bpre.y;
-                    ws->bin[2][rcn & 31] = bpre.z;
+                    ws->bin[rcn & 31] = bpre;
+                    if ((rcn & 31) == 0) ws->bin[32] = bpre;
                     cp_store(io, rcn, qpre);
                     bpre = boundary<PIPE>(ring, rmask, start + rcn + 16, blim, bwf);
                     qpre = query_code(io, start + rcn + 16);
@@ -444,24 +440,33 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             bool fin = false;
             std::integral_constant<bool, true> yes;
             std::integral_constant<bool, false> no;
+            // staging addresses of a 4-step group starting at step g (g % 4 == 0): out entry g&31 + j, in entry
+            // g&31 + 1 + j (<= 32: entry 32 mirrors 0)
+            auto sgo_of = [&](int g) { return sb_out + 16u * (unsigned)(g & 31); };
+            auto sgi_of = [&](int g) { return sb_in + 16u * (unsigned)((g & 31) + 1); };
             if (EAGER && MODE == MODE_INSPECT && top == 0 && t < 32) {
 #pragma unroll 1
-                for (int u = 0; u < 16; ++u)
-                    if (step(yes, yes, t + u, u, u & 3, cbase)) { fin = true; break; }
+                for (int u = 0; u < 16; ++u) {
+                    const int g = t + (u & ~3);
+                    if (step(yes, yes, t + u, u, u & 3, cbase, sgo_of(g), sgi_of(g))) { fin = true; break; }
+                }
             } else if (t + 15 <= span) {
                 // steady state: no lane is past column N during these 16 steps (lanes still left of the strip's
                 // first column compute dead cells: all their inputs are dead and their threshold is >= -(Y+1));
                 // 4-step unrolled body keeps the hot loop inside the instruction cache
 #pragma unroll 1
                 for (int q = 0; q < 16 && !fin; q += 4) {
+                    const unsigned sgo = sgo_of(t + q), sgi = sgi_of(t + q);
 #pragma unroll
                     for (int j = 0; j < 4; ++j)
-                        if (step(no, no, t + q + j, q + j, j, cbase)) { fin = true; break; }
+                        if (step(no, no, t + q + j, q + j, j, cbase, sgo, sgi)) { fin = true; break; }
                 }
             } else {
 #pragma unroll 1
-                for (int u = 0; u < 16; ++u)
-                    if (step(yes, no, t + u, u, u & 3, cbase)) { fin = true; break; }
+                for (int u = 0; u < 16; ++u) {
+                    const int g = t + (u & ~3);
+                    if (step(yes, no, t + u, u, u & 3, cbase, sgo_of(g), sgi_of(g))) { fin = true; break; }
+                }
             }
             if (fin) break;
             t += 16;
@@ -474,7 +479,7 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         if constexpr (MODE == MODE_EXEC) {
             if ((tfinal % SPW) != SPW - 1) io.codes[wbase + (long long)(tfinal / SPW) * 32 + lane] = cw;
         }
-        const int Wtail = ws->bout[2][tfinal & 31];
+        const int Wtail = ws->bout[tfinal & 31].z;
         const int sw = (tfinal / SPW + 1) * 32;
         const bool anyupd = __any_sync(FULL, upd);
         upd = false;
