@@ -67,11 +67,20 @@ typedef struct {
     int32_t ydrop;
     int32_t gapped_threshold;
     int32_t eager_max;
-    int32_t reserved[3];
+    int32_t options;              /* FASTZ_OPT_* bits, 0 = the paper's full design (see below) */
+    int32_t reserved[2];
     void *(*dev_alloc)(size_t bytes, void *stream, void *user);
     void (*dev_free)(void *ptr, void *stream, void *user);
     void *alloc_user;
 } fastz_params;
+
+/* options: ablation switches mirroring the paper's Fig. 9 study and the downstream-output mode.
+ * Results (scores, endpoints, CIGARs) are identical with any FASTZ_OPT_NO_* bit; only the work changes. */
+#define FASTZ_OPT_NO_EAGER 1     /* no eager traceback: every side goes through the executor (P:166-170 off) */
+#define FASTZ_OPT_NO_TRIM 2      /* executor recomputes the whole explored region, not [0,i*]x[0,j*] (P:172 off) */
+#define FASTZ_OPT_NO_BINNING 4   /* one executor queue, warp per side, no length order (P:209-211 off) */
+#define FASTZ_OPT_NO_BLOCK 8     /* no block-per-side scheduling of long sides (inspector and executor) */
+#define FASTZ_OPT_TRACEBACK_ABOVE_K 16 /* traceback only seeds with score >= K; others get an empty CIGAR */
 
 /* A seed is a cut point: the right extension starts at T[tpos], Q[qpos]; the left one at T[tpos-1],
  * Q[qpos-1] going backwards.  0 <= tpos <= tlen, 0 <= qpos <= qlen. */
@@ -83,6 +92,7 @@ typedef struct {
 #define FASTZ_FLAG_LEFT_EAGER 2u  /* left side traced back eagerly in the inspector */
 #define FASTZ_FLAG_RIGHT_EAGER 4u /* right side traced back eagerly */
 #define FASTZ_FLAG_OVERFLOW 8u  /* a one-sided peak score reached 2^29 */
+#define FASTZ_FLAG_NO_CIGAR 16u /* CIGAR skipped (FASTZ_OPT_TRACEBACK_ABOVE_K and score < K) */
 
 /* One alignment per seed, in seed order (64 bytes). */
 typedef struct {

@@ -51,7 +51,7 @@ struct fastz_ctx {
     DevParams dp{};
     int tlen = 0, qlen = 0;
     DBuf Tf, Tr, Qf, Qr, stage;
-    DBuf seeds, score, ti, qj, flags, eops, bound, maxsw, esc;
+    DBuf seeds, score, ti, qj, flags, eops, bound, maxsw, esc, nstrip;
     DBuf woff, soff, roff, bin, list, counters, totals, tmpa, tmpb, tmpc, scan_tmp, wl, wlo;
     DBuf codes, stab, runs, nruns, ciglen, cigar, recs, cells, ring, small;
     int R = 4, grid = 0, nslots = 0, rmask = 0;
@@ -185,6 +185,7 @@ SideArrays make_sides(fastz_ctx* c) {
     s.eops = P_<unsigned long long>(c->eops);
     s.bound = P_<long long>(c->bound);
     s.maxsw = P_<int>(c->maxsw);
+    s.nstrip = P_<int>(c->nstrip);
     return s;
 }
 
@@ -262,7 +263,7 @@ void fastz_destroy(fastz_ctx* c) {
     cudaSetDevice(c->device);
     if (c->stream) cudaStreamSynchronize(c->stream);
     DBuf* bufs[] = {&c->Tf, &c->Tr, &c->Qf, &c->Qr, &c->stage, &c->seeds, &c->score, &c->ti, &c->qj,
-                    &c->flags, &c->eops, &c->bound, &c->maxsw, &c->esc, &c->woff, &c->soff, &c->roff, &c->bin, &c->list,
+                    &c->flags, &c->eops, &c->bound, &c->maxsw, &c->esc, &c->nstrip, &c->woff, &c->soff, &c->roff, &c->bin, &c->list,
                     &c->counters, &c->totals, &c->tmpa, &c->tmpb, &c->tmpc, &c->scan_tmp, &c->wl, &c->wlo, &c->codes,
                     &c->stab, &c->runs, &c->nruns, &c->ciglen, &c->cigar, &c->recs, &c->cells, &c->ring,
                     &c->small};
@@ -311,6 +312,7 @@ int fastz_create(const fastz_params* p, const char* target, int64_t tlen, const 
         c->dp.fold_oe = fold ? 1 : 0;
         c->dp.one = 1;
         c->dp.zero = 0;
+        c->dp.options = p->options;
     }
     c->dp.O = p->gap_open;
     c->dp.E = p->gap_extend;
@@ -359,6 +361,7 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     AL(bound, std::max<int64_t>(ns, 1) * 8);
     AL(maxsw, std::max<int64_t>(ns, 1) * 4);
     AL(esc, std::max<int64_t>(ns, 1) * 4);
+    AL(nstrip, std::max<int64_t>(ns, 1) * 4);
     AL(woff, std::max<int64_t>(ns, 1) * 8);
     AL(soff, std::max<int64_t>(ns, 1) * 8);
     AL(roff, std::max<int64_t>(ns, 1) * 8);
@@ -391,11 +394,11 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
 
     SideArrays sa = make_sides(c);
     ExecPlan pl = make_plan(c);
-    const int esc = escalate_strips();
+    const int esc = (c->dp.options & OPT_NO_BLOCK) ? 0 : escalate_strips();
     CK(launch_inspect(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, esc > 0 ? esc : INT_MAX, st));
     if (esc > 0) CK(launch_inspect_block(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, st));
     CK(cudaEventRecord(c->ev[2], st));
-    CK(launch_bin(c->R, sa, (int)ns, pl, c->scan_tmp.p, stb, P_<long long>(c->tmpa), P_<long long>(c->tmpb),
+    CK(launch_bin(c->R, c->dp, sa, (int)ns, pl, c->scan_tmp.p, stb, P_<long long>(c->tmpa), P_<long long>(c->tmpb),
                   P_<long long>(c->tmpc), st));
     CK(cudaEventRecord(c->ev[3], st));
 

@@ -33,7 +33,8 @@ constexpr int CP_RING = 128;      // column-profile ring entries per warp (+16 m
 constexpr int EAGER_W = 17;       // eager code window: rows/cols 0..16 (16x16)
 
 // side flags
-constexpr uint32_t SF_EAGER = 1u, SF_OVERFLOW = 2u, SF_RING = 4u, SF_ESCALATE = 8u;
+constexpr uint32_t SF_EAGER = 1u, SF_OVERFLOW = 2u, SF_RING = 4u, SF_ESCALATE = 8u, SF_NOTB = 16u;
+constexpr int OPT_NO_EAGER = 1, OPT_NO_TRIM = 2, OPT_NO_BINNING = 4, OPT_NO_BLOCK = 8, OPT_TB_ABOVE_K = 16;
 
 struct DevParams {
     int cp[10];        // column profile per query base b (0..3) and the origin profile (b = 4):
@@ -43,6 +44,7 @@ struct DevParams {
     int K, eager_max;
     int fold_oe;       // O+E folded into the profile (H = X_diag + v) -- see cp above
     int one, zero;     // runtime 1 and 0: keep adds/selects as IMAD on the FMA pipe (ALU pipe is the limiter)
+    int options;       // FASTZ_OPT_* (fastz.h)
 };
 
 // d = a * one + c on the FMA pipe (one == 1 at run time; ptxas cannot fold it into an ALU IADD3)

@@ -17,6 +17,7 @@ struct SideArrays {
     unsigned long long* eops;  // eager ops, 2 bits each, emission order (peak -> origin)
     long long* bound;    // executor words bound, compact layout (0 for eager sides)
     int* maxsw;          // executor words of the widest strip up to the peak strip (block layout)
+    int* nstrip;         // executor strips (i*/H + 1; all inspected strips under FASTZ_OPT_NO_TRIM)
 };
 
 struct Batch {
@@ -67,7 +68,7 @@ cudaError_t launch_inspect_block(int R, int grid, const DevParams& P, const Batc
 int escalate_strips();  // FASTZ_ESCALATE_STRIPS (default 16; 0 disables block-per-side inspection)
 cudaError_t launch_census(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
                           long long* cells, int* counter, cudaStream_t st);
-cudaError_t launch_bin(int R, const SideArrays& sa, int nsides, const ExecPlan& pl, void* scan_tmp,
+cudaError_t launch_bin(int R, const DevParams& P, const SideArrays& sa, int nsides, const ExecPlan& pl, void* scan_tmp,
                        size_t scan_tmp_bytes, long long* tmp_a, long long* tmp_b, long long* tmp_c,
                        cudaStream_t st);
 size_t scan_tmp_bytes(int n);

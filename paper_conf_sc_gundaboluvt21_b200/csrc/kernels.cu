@@ -148,8 +148,10 @@ __device__ __forceinline__ void write_side(const DevParams& P, const SideArrays&
     sa.qj[side] = o.bj;
     sa.flags[side] = flags | ((uint32_t)nops << 8);
     sa.eops[side] = ops;
-    sa.bound[side] = (flags & SF_EAGER) ? 0 : o.bound_words;
-    sa.maxsw[side] = (flags & SF_EAGER) ? 0 : o.bound_maxsw;
+    const bool notrim = P.options & OPT_NO_TRIM;  // executor redoes every explored strip (ablation, P:172 off)
+    sa.bound[side] = (flags & SF_EAGER) ? 0 : (notrim ? o.words : o.bound_words);
+    sa.maxsw[side] = (flags & SF_EAGER) ? 0 : (notrim ? o.maxsw_all : o.bound_maxsw);
+    sa.nstrip[side] = notrim ? o.nstrips : -1;
 }
 
 // ------------------------------------------------------------------------------------------------- inspector
@@ -184,7 +186,8 @@ __global__ void __launch_bounds__(WARPS * 32) k_inspect(DevParams P, Batch b, in
                 uint32_t flags = o.flags;
                 unsigned long long ops = 0;
                 int nops = 0;
-                if (o.bi <= P.eager_max && o.bj <= P.eager_max && !(flags & (SF_RING | SF_OVERFLOW))) {
+                if (o.bi <= P.eager_max && o.bj <= P.eager_max && !(flags & (SF_RING | SF_OVERFLOW)) &&
+                    !(P.options & OPT_NO_EAGER)) {
                     ops = eager_walk(io.ecodes, o.bi, o.bj, nops);
                     flags |= SF_EAGER;
                 }
@@ -272,8 +275,10 @@ __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, in
         io_init(io, sm, ring, rmask, blockIdx.x * WARPS, warp);
         io.ps = &ps;
         setup_side(b, side, io);
-        io.M = sa.ti[side];
-        io.N = sa.qj[side];
+        if (!(P.options & OPT_NO_TRIM)) {  // trimmed executor: the rectangle up to the peak
+            io.M = sa.ti[side];
+            io.N = sa.qj[side];
+        }
         io.codes = out.codes + (pl.woff[side] - base);
         io.stab = out.stab + pl.soff[side];
         io.maxsw = sa.maxsw[side];
@@ -291,8 +296,10 @@ __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, in
         if (idx >= hi) break;
         const int side = pl.list[idx];
         setup_side(b, side, io);
-        io.M = sa.ti[side];
-        io.N = sa.qj[side];
+        if (!(P.options & OPT_NO_TRIM)) {
+            io.M = sa.ti[side];
+            io.N = sa.qj[side];
+        }
         io.codes = out.codes + (pl.woff[side] - base);
         io.stab = out.stab + pl.soff[side];
         SideOut o;
@@ -366,22 +373,27 @@ __device__ __forceinline__ int bin_of(int m) {
 }
 
 template <int R>
-__global__ void k_bin_count(SideArrays sa, int nsides, ExecPlan pl, long long* words, long long* strips,
+__global__ void k_bin_count(DevParams P, SideArrays sa, int nsides, ExecPlan pl, long long* words, long long* strips,
                             long long* runs, int bblock) {
     const int s = blockIdx.x * blockDim.x + threadIdx.x;
     if (s >= nsides) return;
-    const uint32_t fl = sa.flags[s];
-    const bool eager = fl & SF_EAGER;
+    uint32_t fl = sa.flags[s];
+    if ((P.options & OPT_TB_ABOVE_K) && sa.score[s & ~1] + sa.score[s | 1] < P.K) {
+        fl |= SF_NOTB;  // NEXT-3: no traceback below the gapped threshold
+        sa.flags[s] = fl;
+    }
+    const bool skip = fl & (SF_EAGER | SF_NOTB);
     const int ti = sa.ti[s], qj = sa.qj[s];
-    const int bin = eager ? 0 : bin_of(ti > qj ? ti : qj);
+    int bin = skip ? 0 : bin_of(ti > qj ? ti : qj);
+    if (!skip && (P.options & OPT_NO_BINNING)) bin = 1;  // one queue, warp per side (ablation)
     pl.bin[s] = bin;
     atomicAdd(&pl.counters[2 + bin], 1);
     if (fl & SF_RING) atomicOr(&pl.counters[20], 1);
-    const long long ns = ti / (32 * R) + 1;
-    // bins >= 3 run block per side: strip s of the side owns words [s * maxsw, (s + 1) * maxsw)
-    words[s] = eager ? 0 : (bin >= bblock ? ns * (long long)sa.maxsw[s] : sa.bound[s]);
-    strips[s] = eager ? 0 : ns;
-    runs[s] = eager ? 0 : (long long)ti + qj + 1;
+    const long long ns = sa.nstrip[s] >= 0 ? sa.nstrip[s] : ti / (32 * R) + 1;
+    // bins >= bblock run block per side: strip s of the side owns words [s * maxsw, (s + 1) * maxsw)
+    words[s] = skip ? 0 : (bin >= bblock ? ns * (long long)sa.maxsw[s] : sa.bound[s]);
+    strips[s] = skip ? 0 : ns;
+    runs[s] = skip ? 0 : (long long)ti + qj + 1;
 }
 
 __global__ void k_bin_offsets(ExecPlan pl, int nsides, const long long* words, const long long* strips,
@@ -436,14 +448,14 @@ size_t scan_tmp_bytes(int n) {
     return bytes;
 }
 
-cudaError_t launch_bin(int R, const SideArrays& sa, int nsides, const ExecPlan& pl, void* tmp, size_t tmp_bytes,
-                       long long* words, long long* strips, long long* runs, cudaStream_t st) {
-    const int bb = block_bin();
+cudaError_t launch_bin(int R, const DevParams& P, const SideArrays& sa, int nsides, const ExecPlan& pl, void* tmp,
+                       size_t tmp_bytes, long long* words, long long* strips, long long* runs, cudaStream_t st) {
+    const int bb = (P.options & (OPT_NO_BLOCK | OPT_NO_BINNING)) ? 7 : block_bin();
     cudaError_t e;
     if (nsides > 0) {
         const int g = (nsides + 255) / 256;
-        if (R == 2) k_bin_count<2><<<g, 256, 0, st>>>(sa, nsides, pl, words, strips, runs, bb);
-        else k_bin_count<4><<<g, 256, 0, st>>>(sa, nsides, pl, words, strips, runs, bb);
+        if (R == 2) k_bin_count<2><<<g, 256, 0, st>>>(P, sa, nsides, pl, words, strips, runs, bb);
+        else k_bin_count<4><<<g, 256, 0, st>>>(P, sa, nsides, pl, words, strips, runs, bb);
         size_t b = tmp_bytes;
         if ((e = cub::DeviceScan::ExclusiveSum(tmp, b, strips, pl.soff, nsides, st)) != cudaSuccess) return e;
         b = tmp_bytes;
@@ -473,6 +485,7 @@ struct RunVisitor {
     template <class F>
     __device__ __forceinline__ void visit(int seed, F&& f) const {
         const int L = 2 * seed, Rt = 2 * seed + 1;
+        if ((sa.flags[L] | sa.flags[Rt]) & SF_NOTB) return;  // FASTZ_OPT_TRACEBACK_ABOVE_K
         uint32_t cur = 0xffffffffu;
         long long len = 0;
         auto push = [&](uint32_t op, long long n) {
@@ -573,7 +586,8 @@ __global__ void k_combine_write(DevParams P, Batch b, SideArrays sa, ExecPlan pl
     const bool er = sa.ti[Rt] <= P.eager_max && sa.qj[Rt] <= P.eager_max;
     a.flags = (a.score >= P.K ? FASTZ_FLAG_ABOVE_K : 0u) | (el ? FASTZ_FLAG_LEFT_EAGER : 0u) |
               (er ? FASTZ_FLAG_RIGHT_EAGER : 0u) |
-              (((fl | fr) & SF_OVERFLOW) ? FASTZ_FLAG_OVERFLOW : 0u);
+              (((fl | fr) & SF_OVERFLOW) ? FASTZ_FLAG_OVERFLOW : 0u) |
+              (((fl | fr) & SF_NOTB) ? FASTZ_FLAG_NO_CIGAR : 0u);
     a.t_start = tpos - sa.ti[L];
     a.t_end = tpos + sa.ti[Rt];
     a.q_start = qpos - sa.qj[L];

@@ -93,7 +93,9 @@ struct SideOut {
     long long bound_words;   // inspector: executor words up to the peak strip (compact layout)
     int bound_maxsw;         // inspector: max words of one strip up to the peak strip (block layout)
     long long cells;         // census: explored cells (warp total)
-    long long words;         // executor: words written
+    long long words;         // all strips' words (inspector: the untrimmed executor's storage)
+    int maxsw_all;           // widest strip over all strips
+    int nstrips;             // strips run
 };
 
 template <int R>
@@ -148,7 +150,7 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
     int start = 0, Wleft0 = Wout, lastlive = -1, Emax = -1, Wfar = NEG, nfirst = INT_MAX;
     int best = NEG + 1, bi = INT_MAX, bj = INT_MAX;
     long long cum_words = 0, bound_words = 0, cells = 0;
-    int maxsw = 0, bound_maxsw = 0;
+    int maxsw = 0, bound_maxsw = 0, nstr = 0;
     uint32_t flags = 0;
     bool upd = false;
 
@@ -547,6 +549,7 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             __syncwarp();
             if (over) break;
         } else {
+            nstr = s + 1;
             if (over) break;
             lastlive = blast;
             nfirst = bfirst;
@@ -589,6 +592,8 @@ side_done:
         bound_words = ps->bound_words;
         bound_maxsw = ps->bound_maxsw;
         cum_words = ps->cum_words;
+        maxsw = ps->maxsw;
+        nstr = ps->end_strip + 1;
     }
     if constexpr (MODE == MODE_CENSUS) {
 #pragma unroll
@@ -602,6 +607,8 @@ side_done:
     out.bound_maxsw = bound_maxsw;
     out.cells = cells;
     out.words = cum_words;
+    out.maxsw_all = maxsw;
+    out.nstrips = nstr;
 }
 
 // Reset the block-per-problem shared state before a side (one thread; caller synchronises the CTA).

@@ -19,7 +19,8 @@ LIB_PATH = os.path.join(HERE, "libfastz.so")
 
 FASTZ_OK, FASTZ_EINVAL, FASTZ_EBASE, FASTZ_ERANGE = 0, -1, -2, -3
 FASTZ_ENOMEM, FASTZ_ECUDA, FASTZ_ETRUNC, FASTZ_ESTATE = -4, -5, -6, -7
-FLAG_ABOVE_K, FLAG_LEFT_EAGER, FLAG_RIGHT_EAGER, FLAG_OVERFLOW = 1, 2, 4, 8
+FLAG_ABOVE_K, FLAG_LEFT_EAGER, FLAG_RIGHT_EAGER, FLAG_OVERFLOW, FLAG_NO_CIGAR = 1, 2, 4, 8, 16
+OPT_NO_EAGER, OPT_NO_TRIM, OPT_NO_BINNING, OPT_NO_BLOCK, OPT_TRACEBACK_ABOVE_K = 1, 2, 4, 8, 16
 
 # names declared in include/fastz.h (checked by tests/test_abi.py against the header)
 EXPORTS = ["fastz_default_params", "fastz_create", "fastz_extend_seeds", "fastz_get_alignments",
@@ -36,7 +37,8 @@ class FastzError(RuntimeError):
 class fastz_params(ctypes.Structure):
     _fields_ = [("sub", ctypes.c_int32 * 16), ("gap_open", ctypes.c_int32), ("gap_extend", ctypes.c_int32),
                 ("ydrop", ctypes.c_int32), ("gapped_threshold", ctypes.c_int32), ("eager_max", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 3), ("dev_alloc", ctypes.c_void_p), ("dev_free", ctypes.c_void_p),
+                ("options", ctypes.c_int32), ("reserved", ctypes.c_int32 * 2), ("dev_alloc", ctypes.c_void_p),
+                ("dev_free", ctypes.c_void_p),
                 ("alloc_user", ctypes.c_void_p)]
 
 

@@ -205,3 +205,34 @@ def test_executor_waves_under_pool_budget(monkeypatch):
     Q = mutate(rng, T, sub=0.08, indel=0.01)
     bad, *_ = compare(T, Q, [(3000, int(len(Q) * 0.5)), (0, 0), (6000, len(Q)), (10, 10)], census=False)
     assert_ok(bad)
+
+
+@pytest.mark.parametrize("opt", [1, 2, 4, 8, 1 | 2 | 4 | 8])
+def test_ablation_options_do_not_change_results(opt):
+    """FASTZ_OPT_NO_EAGER / NO_TRIM / NO_BINNING / NO_BLOCK (the paper's Fig. 9 variants) change
+    only the work, never the alignments."""
+    w = genome.small_pair(70, length=30000, n_seeds=200)
+    rng = random.Random(71)
+    T = rseq(rng, 5000)
+    Q = mutate(rng, T, sub=0.08, indel=0.01)
+    for TT, QQ, seeds in ((w.T, w.Q, w.seeds), (T, Q, [(2500, int(len(Q) * 0.5)), (0, 0), (5000, len(Q))])):
+        bad, *_ = compare(TT, QQ, seeds, census=False, options=opt)
+        assert_ok(bad)
+
+
+def test_traceback_above_k_only():
+    """FASTZ_OPT_TRACEBACK_ABOVE_K (NEXT-3): seeds below K keep score and endpoints but get no CIGAR."""
+    from paper_conf_sc_gundaboluvt21_b200 import fastz as fz
+    w = genome.small_pair(72, length=30000, n_seeds=300)
+    g0, *_ = run_both(w.T, w.Q, w.seeds)
+    with fz.Aligner(w.T, w.Q, fz.fastz_default_params(options=fz.OPT_TRACEBACK_ABOVE_K)) as al:
+        g1 = al.extend(w.seeds)
+    for f in ("score", "t_start", "t_end", "q_start", "q_end"):
+        assert np.array_equal(g0.rec[f], g1.rec[f])
+    above = g0.rec["score"] >= 3000
+    assert above.any() and (~above).any()
+    for s in range(len(w.seeds)):
+        if above[s]:
+            assert g1.cigar_of(s) == g0.cigar_of(s)
+        else:
+            assert g1.rec["cigar_len"][s] == 0 and g1.rec["flags"][s] & fz.FLAG_NO_CIGAR
