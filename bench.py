@@ -67,6 +67,10 @@ def workload(config: int, n_per_gpu: int, world: int, rank: int):
         n = n_per_gpu or (1 << 20)
         w = genome.config5(n_seeds=n * world)
         desc = "C5: extension-length stress sweep 32 bp - 64 kbp"
+    elif config == 6:
+        n = n_per_gpu or (1 << 20)
+        w = genome.config6(n_seeds=n * world)
+        desc = "C6 (NEXT-2): dissimilar 10 Mbp pair, diverged short homology (cross-genus analog, P:331-340)"
     elif config == 3:
         n = n_per_gpu or (1 << 21)
         w = genome.config3(n_seeds=n * world)

@@ -148,7 +148,7 @@ def _junk_seeds(rng, Tc, Qc, n, homologous_q: np.ndarray | None, index_limit: in
 
 
 def planted_pair(config_id: int, length: int, classes: list, quotas: dict, n_seeds: int,
-                 index_limit: int | None = None, name: str = "") -> Workload:
+                 index_limit: int | None = None, name: str = "", mut_kw: dict | None = None) -> Workload:
     """Random T, Q of ``length`` bp with planted mutated copies T -> Q.
 
     classes: list of (class_name, lo_len, hi_len, count); quotas: class_name -> fraction of seeds
@@ -168,7 +168,7 @@ def planted_pair(config_id: int, length: int, classes: list, quotas: dict, n_see
     per_class = {ci + 1: [] for ci in range(len(classes))}
     for b in range(len(lens)):
         t0, q0, ln = int(tstart[b]), int(qstart[b]), int(lens[b])
-        copy, mapping, clean = mut(rng, Tc[t0:t0 + ln])
+        copy, mapping, clean = mut(rng, Tc[t0:t0 + ln], **(mut_kw or {}))
         copy = copy[: length - q0]
         Qc[q0:q0 + len(copy)] = copy
         hom_q[q0:q0 + len(copy)] = True
@@ -299,7 +299,18 @@ def small_pair(seed: int, length: int = 20_000, n_seeds: int = 256, homology: fl
     return planted_pair(1000 + seed, length, classes, quotas, n_seeds, name=f"small{seed}")
 
 
-CONFIGS = {1: config1, 2: config2, 3: config3, 4: config4, 5: config5}
+def config6(n_seeds: int = 1 << 20) -> Workload:
+    """Dissimilar (cross-genus-like) 10 Mbp pair (NEXT-2; PAPER.md 5.4: "no alignment falls in the two
+    largest size bins"): planted blocks are diverged copies (25% substitutions, 3% indels) of at most 2 kbp,
+    so the seed mix is almost all chance matches and short, low-identity homology."""
+    rng_len = 10_000_000
+    classes = [("S1", 24, 128, 20000), ("S2", 128, 512, 1000), ("M", 512, 2000, 200)]
+    quotas = {"junk": 0.97, "S1": 0.022, "S2": 0.006, "M": 0.002}
+    w = planted_pair(6, rng_len, classes, quotas, n_seeds, name="C6-dissimilar-10Mbp", mut_kw=dict(p_sub=0.25, p_del=0.015, p_ins=0.015))
+    return w
+
+
+CONFIGS = {1: config1, 2: config2, 3: config3, 4: config4, 5: config5, 6: config6}
 
 
 def make(config_id: int, **kw) -> Workload:
