@@ -632,9 +632,14 @@ int inspector_blocks_per_sm(int R) { return R == 2 ? bps_of<2>() : bps_of<4>(); 
         }                                                                                \
     } while (0)
 
+// Inspector escalation of long sides to the block-per-side inspector (FASTZ_ESCALATE_STRIPS, strips; 0 = off).
+// Off by default: measured on C1/C2/C3/C5 (profiles/r1_escalation.jsonl) the pipelined block schedule is slower
+// than independent warps whenever there are more long sides than warps or none at all -- the inspector cannot
+// know lengths in advance, and the warp-per-side queue already hides the long tail.  The executor, which
+// knows the lengths, runs bins >= 3 block per side (FASTZ_BLOCK_BIN).
 int escalate_strips() {  // read per call: tests and ablations switch it at run time
     const char* e = getenv("FASTZ_ESCALATE_STRIPS");
-    int v = e ? atoi(e) : 16;
+    int v = e ? atoi(e) : 0;
     return v < 0 ? 0 : v;
 }
 
