@@ -312,6 +312,9 @@ __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, in
 // ------------------------------------------------------------------------------------------------- traceback
 // One thread per executed side (inter-seed traceback parallelism).  Walks the 4-bit codes from
 // (i*, j*) in state S to the origin; emits run-length ops (len << 2 | op) in peak -> origin order.
+#ifndef TB_PREFETCH
+#define TB_PREFETCH 32
+#endif
 template <int R>
 __global__ void k_traceback(SideArrays sa, ExecPlan pl, int lo, int hi, long long base, Outputs out) {
     constexpr int H = 32 * R, SPW = 8 / R;
@@ -332,30 +335,41 @@ __global__ void k_traceback(SideArrays sa, ExecPlan pl, int lo, int hi, long lon
             len = 1;
         }
     };
+    // the walk is a chain of dependent loads: cache the strip entry and the current code word, and prefetch
+    // the word a few diagonal steps ahead (the common direction) into L1
+    int scur = -1;
+    int2 st = make_int2(0, 0);
+    long long wcur = -1;
+    uint32_t w = 0;
     while (i > 0 || j > 0) {
         const int s = i / H, lr = i - s * H, ln = lr / R, k = lr - ln * R;
-        const int2 st = stab[s];
+        if (s != scur) {
+            st = stab[s];
+            scur = s;
+        }
         const int t = j - st.x + ln;
-        const uint32_t w = codes[(long long)st.y + (long long)(t / SPW) * 32 + ln];
-        const uint32_t code = (w >> ((((t % SPW) * R) + k) * 4)) & 15u;
-        if (state == 0) {
-            const uint32_t src = code & 3u;
-            if (src == 0) {
-                emit(OP_M);
-                --i; --j;
-                continue;
+        const long long wi = (long long)st.y + (long long)(t / SPW) * 32 + ln;
+        if (wi != wcur) {
+            w = codes[wi];
+            wcur = wi;
+            // ~HBM latency / (cycles per step): 32 diagonal steps = 16 lines ahead, within this strip
+            const int i2 = i - TB_PREFETCH, j2 = j - TB_PREFETCH;
+            if (i2 >= s * H && j2 >= st.x) {
+                const int l2 = (i2 - s * H) / R;
+                const long long w2 = (long long)st.y + (long long)((j2 - st.x + l2) / SPW) * 32 + l2;
+                asm volatile("prefetch.global.L2 [%0];" ::"l"(codes + w2));
             }
-            state = (int)src;
         }
-        if (state == 1) {
-            emit(OP_D);
-            state = (code >> 2) & 1u ? 1 : 0;
-            --i;
-        } else {
-            emit(OP_I);
-            state = (code >> 3) & 1u ? 2 : 0;
-            --j;
-        }
+        const uint32_t code = (w >> ((((t % SPW) * R) + k) * 4)) & 15u;
+        // branch-free step (the 32 walks of a warp diverge otherwise): in state S the cell's source decides
+        // (H -> M, D -> enter D, I -> enter I), in a gap state the move is the gap's; one op per iteration
+        const int eff = state == 0 ? (int)(code & 3u) : state;  // 0 M, 1 D, 2 I
+        const uint32_t op = eff == 0 ? (uint32_t)OP_M : (eff == 1 ? (uint32_t)OP_D : (uint32_t)OP_I);
+        const bool ext = eff == 1 ? ((code >> 2) & 1u) : ((code >> 3) & 1u);
+        state = eff == 0 ? 0 : (ext ? eff : 0);
+        i -= eff != 2;
+        j -= eff != 1;
+        emit(op);
     }
     if (len) runs[nr++] = (len << 2) | cur;
     out.nruns[side] = nr;

@@ -39,6 +39,9 @@ namespace fz {
 
 enum { MODE_INSPECT = 0, MODE_EXEC = 1, MODE_CENSUS = 2 };
 
+#ifndef STEADY_UNROLL
+#define STEADY_UNROLL 4  // steps per unrolled steady-state body (4 or 8; 16 overflows the I-cache)
+#endif
 constexpr int PIPE_SLOTS = 8;  // 2K slots for K = 4 warps: a slot is reused only after its consumer finished
 
 struct WarpSmem {
@@ -457,11 +460,15 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                 // first column compute dead cells: all their inputs are dead and their threshold is >= -(Y+1));
                 // 4-step unrolled body keeps the hot loop inside the instruction cache
 #pragma unroll 1
-                for (int q = 0; q < 16 && !fin; q += 4) {
-                    const unsigned sgo = sgo_of(t + q), sgi = sgi_of(t + q);
+                for (int q = 0; q < 16 && !fin; q += STEADY_UNROLL) {
 #pragma unroll
-                    for (int j = 0; j < 4; ++j)
-                        if (step(no, no, t + q + j, q + j, j, cbase, sgo, sgi)) { fin = true; break; }
+                    for (int h = 0; h < STEADY_UNROLL; h += 4) {
+                        const unsigned sgo = sgo_of(t + q + h), sgi = sgi_of(t + q + h);
+#pragma unroll
+                        for (int j = 0; j < 4; ++j)
+                            if (step(no, no, t + q + h + j, q + h + j, j, cbase, sgo, sgi)) { fin = true; break; }
+                        if (fin) break;
+                    }
                 }
             } else {
 #pragma unroll 1
