@@ -1,0 +1,90 @@
+"""C-ABI behaviour on the GPU: input forms (host/device, lowercase), error codes and buffer protocols."""
+import ctypes
+
+import numpy as np
+import pytest
+import torch
+
+from paper_conf_sc_gundaboluvt21_b200 import fastz
+from synth import genome
+
+pytestmark = pytest.mark.gpu
+
+
+def _w():
+    return genome.small_pair(80, length=12000, n_seeds=100)
+
+
+def test_lowercase_equals_uppercase():
+    w = _w()
+    with fastz.Aligner(w.T, w.Q) as a, fastz.Aligner(w.T.lower(), w.Q.lower()) as b:
+        ra, rb = a.extend(w.seeds), b.extend(w.seeds)
+    assert np.array_equal(ra.rec, rb.rec) and ra.cigar == rb.cigar
+
+
+def test_device_sequences_and_device_seeds_equal_host():
+    w = _w()
+    T = torch.frombuffer(bytearray(w.T), dtype=torch.uint8).cuda()
+    Q = torch.frombuffer(bytearray(w.Q), dtype=torch.uint8).cuda()
+    with fastz.Aligner(w.T, w.Q) as a, fastz.Aligner(T, Q) as b:
+        ra = a.extend(w.seeds)
+        rb = b.extend(torch.from_numpy(w.seeds).cuda())
+    assert np.array_equal(ra.rec, rb.rec) and ra.cigar == rb.cigar
+
+
+def test_invalid_base_reports_index():
+    with pytest.raises(fastz.FastzError) as e:
+        fastz.Aligner(b"ACGTNACGT", b"ACGT")
+    assert e.value.status == fastz.FASTZ_EBASE and "index 4" in str(e.value)
+    with pytest.raises(fastz.FastzError) as e:
+        fastz.Aligner(b"ACGT", b"AC-T")
+    assert e.value.status == fastz.FASTZ_EBASE
+
+
+def test_seed_out_of_range():
+    with fastz.Aligner(b"ACGTACGT", b"ACGTACGT") as a:
+        with pytest.raises(fastz.FastzError) as e:
+            a.extend(np.array([[1, 1], [9, 2]], np.int64))
+        assert e.value.status == fastz.FASTZ_ERANGE and "seed 1" in str(e.value)
+        with pytest.raises(fastz.FastzError):
+            a.extend(np.array([[-1, 0]], np.int64))
+
+
+def test_estate_and_etrunc():
+    L = fastz.lib()
+    w = _w()
+    ctx = fastz.fastz_create(fastz.fastz_default_params(), w.T, w.Q, 0)
+    try:
+        n, nb = ctypes.c_int64(), ctypes.c_int64()
+        assert L.fastz_get_alignments(ctx, None, 0, None, 0, ctypes.byref(n), ctypes.byref(nb)) == fastz.FASTZ_ESTATE
+        fastz.fastz_extend_seeds(ctx, w.seeds)
+        rc = L.fastz_get_alignments(ctx, None, 0, None, 0, ctypes.byref(n), ctypes.byref(nb))
+        assert rc == fastz.FASTZ_ETRUNC and n.value == len(w.seeds) and nb.value > 0
+        rec = np.zeros(n.value, dtype=fastz.ALIGN_DTYPE)
+        small = ctypes.create_string_buffer(nb.value - 1)
+        rc = L.fastz_get_alignments(ctx, rec.ctypes.data, n.value, small, nb.value - 1, ctypes.byref(n), ctypes.byref(nb))
+        assert rc == fastz.FASTZ_ETRUNC
+        full = ctypes.create_string_buffer(nb.value)
+        assert L.fastz_get_alignments(ctx, rec.ctypes.data, n.value, full, nb.value, ctypes.byref(n),
+                                      ctypes.byref(nb)) == 0
+        recs, cig = ctypes.c_void_p(), ctypes.c_void_p()
+        assert L.fastz_get_alignments_device(ctx, ctypes.byref(recs), ctypes.byref(cig), ctypes.byref(n),
+                                             ctypes.byref(nb)) == 0
+        assert recs.value and cig.value
+    finally:
+        fastz.fastz_destroy(ctx)
+
+
+def test_repeated_batches_reuse_context():
+    w = _w()
+    with fastz.Aligner(w.T, w.Q) as a:
+        r1 = a.extend(w.seeds)
+        r2 = a.extend(w.seeds[:10])
+        r3 = a.extend(w.seeds)
+    assert np.array_equal(r1.rec, r3.rec) and r1.cigar == r3.cigar
+    assert np.array_equal(r2.rec[:10]["score"], r1.rec[:10]["score"])
+
+
+def test_int_peak_is_sane():
+    ops, mhz = fastz.fastz_int_peak(0, 50.0)
+    assert 1e12 < ops < 1e14 and 500 < mhz < 3000

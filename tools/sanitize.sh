@@ -1,0 +1,17 @@
+# compute-sanitizer on a small mixed workload (memcheck, racecheck, synccheck, initcheck); block-per-side forced
+mkdir -p gpurun_out
+python -m paper_conf_sc_gundaboluvt21_b200.build > /dev/null
+cat > /tmp/san_case.py <<'PY'
+import os, sys
+sys.path.insert(0, os.getcwd())
+from synth import genome
+from paper_conf_sc_gundaboluvt21_b200 import fastz
+w = genome.small_pair(90, length=8000, n_seeds=40)
+with fastz.Aligner(w.T, w.Q) as a:
+    r = a.extend(w.seeds)
+    a.census()
+print("ok", len(r.rec))
+PY
+for tool in memcheck racecheck synccheck initcheck; do
+  FASTZ_ESCALATE_STRIPS=2 FASTZ_BLOCK_BIN=1 timeout 900 compute-sanitizer --tool $tool --error-exitcode 9 python /tmp/san_case.py > gpurun_out/san_$tool.log 2>&1; echo "$tool rc=$?"; tail -2 gpurun_out/san_$tool.log
+done
