@@ -37,9 +37,10 @@ def to_ascii(codes: np.ndarray) -> bytes:
     return ASCII[codes].tobytes()
 
 
-def mut(rng, src: np.ndarray, p_del=0.005, p_ins=0.005, p_sub=0.10):
+def mut(rng, src: np.ndarray, p_del=0.005, p_ins=0.005, p_sub=0.10, return_starts=False):
     """Mutated copy of ``src`` and the map source index -> copy index (-1 if deleted) and a mask of
-    source bases that survive unsubstituted with no insertion in front of them."""
+    source bases that survive unsubstituted with no insertion in front of them (and, optionally, the copy
+    position where each source base's contribution starts)."""
     n = len(src)
     u = rng.random(n)
     dele = u < p_del
@@ -56,6 +57,8 @@ def mut(rng, src: np.ndarray, p_del=0.005, p_ins=0.005, p_sub=0.10):
     out[pos[keep]] = val[keep]
     mapping = np.where(keep, pos, -1)
     clean = keep & ~subs & ~ins
+    if return_starts:
+        return out, mapping, clean, starts
     return out, mapping, clean
 
 
@@ -107,12 +110,17 @@ def _layout(rng, total: int, lengths: np.ndarray) -> np.ndarray:
     assert free > 0, "blocks do not fit"
     order = rng.permutation(len(lengths))
     cuts = np.sort(rng.integers(0, free, len(lengths)))
+    lo = lengths[order]
     starts = np.empty(len(lengths), dtype=np.int64)
-    off = 0
-    for rank, b in enumerate(order):
-        starts[b] = cuts[rank] + off
-        off += int(lengths[b])
+    starts[order] = cuts + np.concatenate([[0], np.cumsum(lo)[:-1]]).astype(np.int64)
     return starts
+
+
+def _ranges(starts: np.ndarray, lens: np.ndarray) -> np.ndarray:
+    """Concatenation of [starts[b], starts[b] + lens[b]) for all b (vectorised)."""
+    tot = int(lens.sum())
+    base = np.repeat(starts - np.concatenate([[0], np.cumsum(lens)[:-1]]), lens)
+    return base + np.arange(tot, dtype=np.int64)
 
 
 def _loguniform(rng, lo, hi, n):
@@ -164,18 +172,32 @@ def planted_pair(config_id: int, length: int, classes: list, quotas: dict, n_see
     cls = np.concatenate(cls)
     tstart = _layout(rng, length, lens + 64)
     qstart = _layout(rng, length, lens + 64)
+    # mutate every block in one pass (mut is per-base independent), then split by block
+    bsrc = np.concatenate([[0], np.cumsum(lens)[:-1]]).astype(np.int64)  # block start in the concatenation
+    src = Tc[_ranges(tstart, lens)]
+    copy, mapping, clean, ostart = mut(rng, src, return_starts=True, **(mut_kw or {}))
+    ostart = np.append(ostart, len(copy))
+    ob = ostart[bsrc]                                   # block's first position in `copy`
+    olen = ostart[bsrc + lens] - ob                     # block's copy length
+    qpos = _ranges(qstart, olen)
+    keep = qpos < length
+    Qc[qpos[keep]] = copy[keep]
     hom_q = np.zeros(length, dtype=bool)
+    hom_q[qpos[keep]] = True
+    # exact 12-mers on each block's true alignment (not crossing block boundaries, inside the sequence)
+    ks = exact_kmer_starts(mapping, clean)
+    blk = np.searchsorted(bsrc, ks, side="right") - 1
+    inside = (ks + K <= bsrc[blk] + lens[blk]) & (mapping[ks] + K <= ob[blk] + olen[blk])
+    ks, blk = ks[inside], blk[inside]
+    tcoord = tstart[blk] + (ks - bsrc[blk]) + K // 2
+    qcoord = qstart[blk] + (mapping[ks] - ob[blk]) + K // 2
+    okq = qcoord + K // 2 <= length
+    ks, blk, tcoord, qcoord = ks[okq], blk[okq], tcoord[okq], qcoord[okq]
     per_class = {ci + 1: [] for ci in range(len(classes))}
-    for b in range(len(lens)):
-        t0, q0, ln = int(tstart[b]), int(qstart[b]), int(lens[b])
-        copy, mapping, clean = mut(rng, Tc[t0:t0 + ln], **(mut_kw or {}))
-        copy = copy[: length - q0]
-        Qc[q0:q0 + len(copy)] = copy
-        hom_q[q0:q0 + len(copy)] = True
-        ks = exact_kmer_starts(mapping, clean)
-        ks = ks[mapping[ks] + K <= len(copy)]
-        if len(ks):
-            per_class[int(cls[b])].append(np.stack([t0 + ks + K // 2, q0 + mapping[ks] + K // 2], axis=1))
+    for ci in range(len(classes)):
+        m = cls[blk] == ci + 1
+        if m.any():
+            per_class[ci + 1].append(np.stack([tcoord[m], qcoord[m]], axis=1))
     seeds, klass = [], []
     counts = {nm: int(round(quotas.get(nm, 0.0) * n_seeds)) for nm in ["junk"] + [c[0] for c in classes]}
     counts["junk"] += n_seeds - sum(counts.values())
