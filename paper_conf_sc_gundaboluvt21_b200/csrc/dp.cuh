@@ -83,6 +83,14 @@ __device__ __forceinline__ void ld_shared4_if(bool p, unsigned addr, int4& v) {
                  : "r"((unsigned)p), "r"(addr));
 }
 
+// predicated 128-bit shared load into three fresh registers (4th word discarded)
+__device__ __forceinline__ void ld_shared3_if(bool p, unsigned addr, int& x, int& y, int& z) {
+    int pad;
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %4, 0; @q ld.shared.v4.b32 {%0, %1, %2, %3}, [%5]; }"
+                 : "+r"(x), "+r"(y), "+r"(z), "=r"(pad)
+                 : "r"((unsigned)p), "r"(addr));
+}
+
 __device__ __forceinline__ int prmt(int a, int b, int s) {
     int d;
     asm("prmt.b32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(s));

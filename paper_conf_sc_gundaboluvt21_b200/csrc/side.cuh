@@ -142,6 +142,7 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
     WarpSmem* __restrict__ ws = io.ws;
     PipeShared* __restrict__ ps = io.ps;
     const bool is31 = lane == 31;
+    const bool is0 = lane == 0;
     const unsigned sb_in = (unsigned)__cvta_generic_to_shared(&ws->bin[0]);
     const unsigned sb_out = (unsigned)__cvta_generic_to_shared(&ws->bout[0]);
 
@@ -272,7 +273,6 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             qpre = query_code(io, start + 32 + lane);
         }
         __syncwarp();
-        if (lane == 31) bq = ws->bin[0];
         uint32_t cw = 0;
         int lastlive_t = -1;  // last 4-step group end at which this lane had a live cell (termination)
         int cacc = NEG;       // max X of this lane over the current 4-step group
@@ -320,6 +320,8 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             int xu = __shfl_sync(FULL, bq.x, src);
             int du = __shfl_sync(FULL, bq.y, src);
             int wu = __shfl_sync(FULL, bq.z, src);
+            // lane 0 replaces what lane 31 sent with the boundary row for its column (relative column tt)
+            ld_shared3_if(is0, sgi + 16u * (unsigned)j, xu, du, wu);
             int cmv = NEG;
             if (valid) {
                 const int2 cp = ws->cp[cbase + u];
@@ -378,9 +380,8 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                     }
                 }
             }
-            // lane 31 parks its bottom row and picks up the boundary for lane 0's next column
+            // lane 31 parks its bottom row
             st_shared4_if(is31, sgo + 16u * (unsigned)j, bq);
-            ld_shared4_if(is31, sgi + 16u * (unsigned)j, bq);
             if constexpr (MODE == MODE_EXEC) {
                 if ((j % SPW) == SPW - 1) {  // j == tt mod 4 and SPW divides 4
                     io.codes[wbase + (long long)(tt / SPW) * 32 + lane] = cw;
@@ -445,10 +446,9 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             bool fin = false;
             std::integral_constant<bool, true> yes;
             std::integral_constant<bool, false> no;
-            // staging addresses of a 4-step group starting at step g (g % 4 == 0): out entry g&31 + j, in entry
-            // g&31 + 1 + j (<= 32: entry 32 mirrors 0)
+            // staging addresses of a 4-step group starting at step g (g % 4 == 0): out and in entry g&31 + j
             auto sgo_of = [&](int g) { return sb_out + 16u * (unsigned)(g & 31); };
-            auto sgi_of = [&](int g) { return sb_in + 16u * (unsigned)((g & 31) + 1); };
+            auto sgi_of = [&](int g) { return sb_in + 16u * (unsigned)(g & 31); };
             if (EAGER && MODE == MODE_INSPECT && top == 0 && t < 32) {
 #pragma unroll 1
                 for (int u = 0; u < 16; ++u) {
