@@ -29,7 +29,7 @@ constexpr int NEG = -(1 << 30);   // dead score (X space)
 constexpr int BIG = (1 << 30);    // threshold of rows beyond M: nothing there is ever live
 constexpr unsigned FULL = 0xffffffffu;
 constexpr int SCORE_LIMIT = 1 << 29;
-constexpr int CP_RING = 128;      // column-profile ring entries per warp (+16 mirrored)
+constexpr int CP_RING = 128;      // column-profile ring entries per warp (+BLK mirrored)
 constexpr int EAGER_W = 17;       // eager code window: rows/cols 0..16 (16x16)
 
 // side flags

@@ -20,12 +20,13 @@
 //                numerator; not on the timed path.
 //
 // Per-step data movement (the paper's register exchange, re-designed for sm_100a):
-//  * lane l receives the bottom row (X, D, W) of lane l-1 with a ROTATING shuffle (src = l-1 mod 32): lane 0
-//    receives from lane 31, which -- after parking its own bottom row in shared staging -- holds the previous
-//    strip's boundary value for lane 0's next column.  No per-step global memory access, no lane-0 selects.
-//  * every 16 steps the warp moves 16 boundary values global ring -> shared staging (prefetched one block
-//    ahead) and 16 parked bottom-row values shared -> global ring, both coalesced; the parked values also
-//    give the bottom row's first/last live column (next strip's start, termination test).
+//  * lane l receives the bottom row (X, D, W) of lane l-1 with a ROTATING shuffle (src = l-1 mod 32); lane 0
+//    then overwrites what lane 31 sent with the previous strip's boundary value for its column (one predicated
+//    128-bit shared load straight into the shuffle results), and lane 31 parks its own bottom row in shared
+//    staging (one predicated 128-bit store).  No per-step global memory access, no selects.
+//  * every BLK = 32 steps (16 in PIPE) the warp moves 32 boundary values global ring -> shared staging (prefetched into
+//    registers one block ahead) and 32 parked bottom-row values shared -> global ring, both coalesced; the
+//    parked values also give the bottom row's first/last live column (next strip's start, termination test).
 //  * termination: each lane keeps the last step at which one of its R cells was live; the strip is done at
 //    column x (lane 31's) iff no lane has had a live cell since it processed x and the boundary row has no
 //    live cell at or after x -- the unrolled form of the per-lane "done" chain (lane l is done at x iff its
@@ -42,13 +43,15 @@ enum { MODE_INSPECT = 0, MODE_EXEC = 1, MODE_CENSUS = 2 };
 #ifndef STEADY_UNROLL
 #define STEADY_UNROLL 4  // steps per unrolled steady-state body (4 or 8; 16 overflows the I-cache)
 #endif
+// steps per staging block (refill of boundary/profiles, park of the bottom row): BLK for SOLO; PIPE uses 16 so a
+// consumer strip trails its producer by fewer columns (flush granularity + prefetch distance)
+constexpr int BLK = 32;
 constexpr int PIPE_SLOTS = 8;  // 2K slots for K = 4 warps: a slot is reused only after its consumer finished
 
 struct WarpSmem {
-    int2 cp[CP_RING + 16];  // column profiles, ring over relative columns (+16 mirrored)
-    int4 bin[33];           // boundary row staging {X, D, W, -} (lane 0's input, served through lane 31);
-                            // entry 32 mirrors entry 0 so a 4-step group never wraps
-    int4 bout[32];          // lane 31's bottom-row outputs {X, D, W, -} awaiting the global ring
+    int2 cp[CP_RING + BLK]; // column profiles, ring over relative columns (+BLK mirrored)
+    int4 bin[BLK];          // boundary row staging {X, D, W, -}: lane 0's input of the current block
+    int4 bout[BLK];         // lane 31's bottom-row outputs {X, D, W, -} awaiting the global ring
 };
 
 // Block-per-problem (PIPE) shared state of one side.  Strip s owns slot s % PIPE_SLOTS.
@@ -115,7 +118,7 @@ __device__ __forceinline__ void cp_store(const SideIO& io, int rc, int code) {
     const int2 v = io.cptab[code];
     const int idx = rc & (CP_RING - 1);
     io.ws->cp[idx] = v;
-    if (idx < 16) io.ws->cp[idx + CP_RING] = v;
+    if (idx < BLK) io.ws->cp[idx + CP_RING] = v;
 }
 
 // Boundary row value at column c: the ring holds exact entries up to column lim, beyond it the row is dead
@@ -132,7 +135,9 @@ template <int R, int MODE, bool EAGER, bool FOLD, bool PIPE>
 __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, SideOut& out) {
     constexpr int H = StripGeom<R>::H;
     constexpr int SPW = StripGeom<R>::SPW;
+    constexpr int BK = PIPE ? 16 : BLK;
     const int lane = threadIdx.x & 31;
+    const bool stager = BK == 32 || lane < BK;  // lanes that move one staging entry per block
     const int src = (lane + 31) & 31;
     const int M = io.M, N = io.N;
     const int E = P.E, OE = P.OE, OEmY = P.OE - P.Y, mE = -P.E, mOE = -P.OE;
@@ -258,19 +263,15 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                 }
             }
         };
-        pipe_sync(start + 47);
-        // staging: boundary for relative columns [0, 32), column profiles [0, 32); prefetch the next 16
-        {
-            const int4 v = boundary<PIPE>(ring, rmask, start + lane, blim, bwf);
-            ws->bin[lane] = v;
-            if (lane == 0) ws->bin[32] = v;
-        }
-        cp_store(io, lane, query_code(io, start + lane));
+        pipe_sync(start + 2 * BK - 1);
+        // staging: boundary and column profiles for relative columns [0, BK); prefetch the next BK
         int4 bpre = make_int4(NEG, NEG, bwf, 0);
         int qpre = 4;
-        if (lane < 16) {
-            bpre = boundary<PIPE>(ring, rmask, start + 32 + lane, blim, bwf);
-            qpre = query_code(io, start + 32 + lane);
+        if (stager) {
+            ws->bin[lane] = boundary<PIPE>(ring, rmask, start + lane, blim, bwf);
+            cp_store(io, lane, query_code(io, start + lane));
+            bpre = boundary<PIPE>(ring, rmask, start + BK + lane, blim, bwf);
+            qpre = query_code(io, start + BK + lane);
         }
         __syncwarp();
         uint32_t cw = 0;
@@ -280,13 +281,13 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         int bfirst = INT_MAX, blast = -1;  // bottom row's first/last live column (from the parked values)
         if constexpr (PIPE) lastlive = s == 0 ? -1 : INT_MAX;  // unknown until strip s-1 has finished
 
-        // park steps [st0, stmax] (at most 16) of lane 31's outputs in the ring (lanes 0..15); track live columns
+        // park steps [st0, stmax] (at most BK) of lane 31's outputs in the ring; track live columns
         auto park = [&](int st0, int stmax) {
             const int st = st0 + lane, rc31 = st - 31;
-            const bool ok = lane < 16 && st <= stmax && rc31 >= 0 && rc31 <= span;
+            const bool ok = stager && st <= stmax && rc31 >= 0 && rc31 <= span;
             int xv = NEG;
             if (ok) {
-                const int4 v = ws->bout[st & 31];
+                const int4 v = ws->bout[st & (BK - 1)];
                 xv = v.x;
                 ring[(start + rc31) & rmask] = v;
             }
@@ -429,16 +430,15 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         for (;;) {
             if (t > 0) {
                 __syncwarp();  // lane 31's parked rows of the previous block -> visible to lanes 0..15
-                park(t - 16, t - 1);
-                pipe_sync(start + t + 47);
-                // staging refills for relative columns [t+16, t+32), prefetch [t+32, t+48)
-                if (lane < 16) {
-                    const int rcn = t + 16 + lane;
-                    ws->bin[rcn & 31] = bpre;
-                    if ((rcn & 31) == 0) ws->bin[32] = bpre;
+                park(t - BK, t - 1);
+                pipe_sync(start + t + 2 * BK - 1);
+                // staging refill for relative columns [t, t+BK) (prefetched), prefetch [t+BK, t+2BK)
+                if (stager) {
+                    const int rcn = t + lane;
+                    ws->bin[rcn & (BK - 1)] = bpre;
                     cp_store(io, rcn, qpre);
-                    bpre = boundary<PIPE>(ring, rmask, start + rcn + 16, blim, bwf);
-                    qpre = query_code(io, start + rcn + 16);
+                    bpre = boundary<PIPE>(ring, rmask, start + rcn + BK, blim, bwf);
+                    qpre = query_code(io, start + rcn + BK);
                 }
             }
             __syncwarp();
@@ -446,21 +446,21 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             bool fin = false;
             std::integral_constant<bool, true> yes;
             std::integral_constant<bool, false> no;
-            // staging addresses of a 4-step group starting at step g (g % 4 == 0): out and in entry g&31 + j
-            auto sgo_of = [&](int g) { return sb_out + 16u * (unsigned)(g & 31); };
-            auto sgi_of = [&](int g) { return sb_in + 16u * (unsigned)(g & 31); };
+            // staging addresses of a 4-step group starting at step g (g % 4 == 0): out and in entry g%BLK + j
+            auto sgo_of = [&](int g) { return sb_out + 16u * (unsigned)(g & (BK - 1)); };
+            auto sgi_of = [&](int g) { return sb_in + 16u * (unsigned)(g & (BK - 1)); };
             if (EAGER && MODE == MODE_INSPECT && top == 0 && t < 32) {
 #pragma unroll 1
-                for (int u = 0; u < 16; ++u) {
+                for (int u = 0; u < BK; ++u) {
                     const int g = t + (u & ~3);
                     if (step(yes, yes, t + u, u, u & 3, cbase, sgo_of(g), sgi_of(g))) { fin = true; break; }
                 }
-            } else if (t + 15 <= span) {
-                // steady state: no lane is past column N during these 16 steps (lanes still left of the strip's
+            } else if (t + BK - 1 <= span) {
+                // steady state: no lane is past column N during these BK steps (lanes still left of the strip's
                 // first column compute dead cells: all their inputs are dead and their threshold is >= -(Y+1));
                 // 4-step unrolled body keeps the hot loop inside the instruction cache
 #pragma unroll 1
-                for (int q = 0; q < 16 && !fin; q += STEADY_UNROLL) {
+                for (int q = 0; q < BK && !fin; q += STEADY_UNROLL) {
 #pragma unroll
                     for (int h = 0; h < STEADY_UNROLL; h += 4) {
                         const unsigned sgo = sgo_of(t + q + h), sgi = sgi_of(t + q + h);
@@ -472,13 +472,13 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                 }
             } else {
 #pragma unroll 1
-                for (int u = 0; u < 16; ++u) {
+                for (int u = 0; u < BK; ++u) {
                     const int g = t + (u & ~3);
                     if (step(yes, no, t + u, u, u & 3, cbase, sgo_of(g), sgi_of(g))) { fin = true; break; }
                 }
             }
             if (fin) break;
-            t += 16;
+            t += BK;
         }
 
         // ------------------------------------------------------------------ strip finish
@@ -488,7 +488,7 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         if constexpr (MODE == MODE_EXEC) {
             if ((tfinal % SPW) != SPW - 1) io.codes[wbase + (long long)(tfinal / SPW) * 32 + lane] = cw;
         }
-        const int Wtail = ws->bout[tfinal & 31].z;
+        const int Wtail = ws->bout[tfinal & (BK - 1)].z;
         const int sw = (tfinal / SPW + 1) * 32;
         const bool anyupd = __any_sync(FULL, upd);
         upd = false;
