@@ -297,19 +297,13 @@ int fastz_create(const fastz_params* p, const char* target, int64_t tlen, const 
         }
         c->own_stream = true;
     }
-    // column profiles (int16 pairs) per query base; profile 4 = the origin column (sub = 0).  O+E is folded
-    // into the profile when every value still fits int16 (then H = X_diag + v is one FMA-pipe IMAD).
+    // substitution table with O+E folded in (H = X_diag + v is one FMA-pipe IMAD); column code 4 = the origin
+    // column (sub = 0)
     {
         const int oe = p->gap_open + p->gap_extend;
-        bool fold = oe <= 32767;
-        for (int k = 0; k < 16; ++k) fold = fold && (p->sub[k] + oe >= -32768) && (p->sub[k] + oe <= 32767);
-        const int add = fold ? oe : 0;
-        for (int b = 0; b < 4; ++b) {
-            c->dp.cp[2 * b] = ((p->sub[4 * 0 + b] + add) & 0xffff) | ((p->sub[4 * 1 + b] + add) << 16);
-            c->dp.cp[2 * b + 1] = ((p->sub[4 * 2 + b] + add) & 0xffff) | ((p->sub[4 * 3 + b] + add) << 16);
-        }
-        c->dp.cp[8] = c->dp.cp[9] = (add & 0xffff) | (add << 16);
-        c->dp.fold_oe = fold ? 1 : 0;
+        for (int b = 0; b < 4; ++b)
+            for (int a = 0; a < 4; ++a) c->dp.sv[4 * b + a] = p->sub[4 * a + b] + oe;
+        for (int a = 0; a < 4; ++a) c->dp.sv[16 + a] = oe;
         c->dp.one = 1;
         c->dp.zero = 0;
         c->dp.options = p->options;

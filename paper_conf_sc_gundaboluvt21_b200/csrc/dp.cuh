@@ -17,8 +17,9 @@
 // rectangle [0,i]x[0,j], reading R3):  thr = max(W_up, W_left), live iff S >= thr, W = max(thr, S - Y).
 // Only S is killed (dead X = NEG); I and D keep their values -- by the lemma in DESIGN.md (V never decreases
 // along a predecessor edge) this yields the same live set, scores, peak and on-path traceback codes as
-// killing all three.  Substitution scores come from a per-column profile (4 x int16 for the column's query
-// base, streamed through a per-warp shared-memory ring) selected per row with one PRMT.
+// killing all three.  Substitution scores (with O+E folded in) come from a shared-memory table indexed by the
+// column's query code (streamed through a per-warp ring as a byte offset) and the lane's row-pair bases: one
+// conflict-free LDS.64 per row pair and step, no ALU-pipe select.
 #pragma once
 #include <cstdint>
 #include <climits>
@@ -31,18 +32,22 @@ constexpr unsigned FULL = 0xffffffffu;
 constexpr int SCORE_LIMIT = 1 << 29;
 constexpr int CP_RING = 128;      // column-profile ring entries per warp (+BLK mirrored)
 constexpr int EAGER_W = 17;       // eager code window: rows/cols 0..16 (16x16)
+// Substitution table in shared memory: entry e = code * 16 + a0 * 4 + a1 (query code 0..4, target bases of a
+// row pair) holds int2 {sub(a0, code) + O + E, sub(a1, code) + O + E} (code 4 = the origin column: sub = 0),
+// replicated 16x so that the 16 lanes of a half-warp read 16 distinct bank pairs (conflict-free LDS.64).
+constexpr int SUBTAB_REP = 16;
+constexpr int SUBTAB_ENTRY = SUBTAB_REP * 8;    // bytes per entry
+constexpr int SUBTAB_CODE = 16 * SUBTAB_ENTRY;  // bytes per query code
+constexpr int SUBTAB_INTS = 5 * SUBTAB_CODE / 4;
 
 // side flags
 constexpr uint32_t SF_EAGER = 1u, SF_OVERFLOW = 2u, SF_RING = 4u, SF_ESCALATE = 8u, SF_NOTB = 16u;
 constexpr int OPT_NO_EAGER = 1, OPT_NO_TRIM = 2, OPT_NO_BINNING = 4, OPT_NO_BLOCK = 8, OPT_TB_ABOVE_K = 16;
 
 struct DevParams {
-    int cp[10];        // column profile per query base b (0..3) and the origin profile (b = 4):
-                       //   cp[2b] = (v(A,b) & 0xffff) | v(C,b) << 16, cp[2b+1] = (v(G,b) & 0xffff) | v(T,b) << 16
-                       //   with v = sub + O + E when every such value fits int16 (fold_oe = 1), else v = sub
+    int sv[20];        // sv[4b + a] = sub(a, b) + O + E for query base b = 0..3; sv[16 + a] = O + E (origin column)
     int O, E, Y, OE;   // gap open, extend, y-drop, O+E
     int K, eager_max;
-    int fold_oe;       // O+E folded into the profile (H = X_diag + v) -- see cp above
     int one, zero;     // runtime 1 and 0: keep adds/selects as IMAD on the FMA pipe (ALU pipe is the limiter)
     int options;       // FASTZ_OPT_* (fastz.h)
 };
@@ -61,6 +66,11 @@ __device__ __forceinline__ int kill_fma(int s, int thr, int mOE, int one, int ze
     asm("{ .reg .pred p; setp.lt.s32 p, %1, %2; @p mad.lo.s32 %0, %0, %3, %4; }"
         : "+r"(x) : "r"(s), "r"(thr), "r"(zero), "n"(NEG));
     return x;
+}
+
+// 64-bit shared load of two words
+__device__ __forceinline__ void ld_shared2(int addr, int& x, int& y) {
+    asm volatile("ld.shared.v2.b32 {%0, %1}, [%2];" : "=r"(x), "=r"(y) : "r"(addr));
 }
 
 // predicated shared-memory store / load (keeps per-lane staging as predicated instructions, not a branch)
@@ -95,13 +105,6 @@ __device__ __forceinline__ int prmt(int a, int b, int s) {
     int d;
     asm("prmt.b32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(s));
     return d;
-}
-
-// PRMT selector picking the signed int16 sub(a, .) out of a column profile {lo, hi} (bytes 2a, 2a+1,
-// sign-replicated into bytes 2 and 3).
-__device__ __forceinline__ int row_selector(int a) {
-    const int b0 = 2 * a, b1 = 2 * a + 1;
-    return b0 | (b1 << 4) | ((8 | b1) << 8) | ((8 | b1) << 12);
 }
 
 // base k (0-based position pos) of a 2-bit packed sequence (16 bases per word, base 0 in bits 1:0)

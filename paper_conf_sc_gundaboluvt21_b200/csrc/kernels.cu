@@ -84,13 +84,21 @@ __device__ __forceinline__ void setup_side(const Batch& b, int side, SideIO& io)
 constexpr int OP_M = 0, OP_I = 1, OP_D = 2;
 
 struct SmemDP {
+    alignas(16) int subtab[SUBTAB_INTS];
     WarpSmem w[WARPS];
-    int2 cptab[8];
     uint8_t ecodes[WARPS][EAGER_W * EAGER_W + 15];
 };
 
 __device__ __forceinline__ void smem_init(SmemDP& sm, const DevParams& P) {
-    if (threadIdx.x < 5) sm.cptab[threadIdx.x] = make_int2(P.cp[2 * threadIdx.x], P.cp[2 * threadIdx.x + 1]);
+    for (int idx = threadIdx.x; idx < SUBTAB_INTS / 2; idx += blockDim.x) {
+        const int e = idx / SUBTAB_REP, code = e >> 4, a0 = (e >> 2) & 3, a1 = e & 3;
+        sm.subtab[2 * idx] = P.sv[4 * code + a0];
+        sm.subtab[2 * idx + 1] = P.sv[4 * code + a1];
+    }
+    // the column-code ring is read ahead of the strip's first column during ramp-up (dead cells): it must
+    // always hold valid table offsets
+    for (int idx = threadIdx.x; idx < WARPS * (CP_RING + BLK); idx += blockDim.x)
+        sm.w[idx / (CP_RING + BLK)].co[idx % (CP_RING + BLK)] = 4 * SUBTAB_CODE;
     __syncthreads();
 }
 
@@ -98,7 +106,7 @@ __device__ __forceinline__ void io_init(SideIO& io, SmemDP& sm, int4* ring, int 
     io.ring = ring + (size_t)warp_slot * (size_t)(rmask + 1);
     io.rmask = rmask;
     io.ws = &sm.w[warp];
-    io.cptab = sm.cptab;
+    io.subtab = (unsigned)__cvta_generic_to_shared(sm.subtab);
     io.ecodes = sm.ecodes[warp];
     io.eager_max = -1;
     io.codes = nullptr;
@@ -159,7 +167,7 @@ __device__ __forceinline__ void write_side(const DevParams& P, const SideArrays&
 // 32 CUDA streams).  Score-only DP + eager 17x17 corner codes; when the peak lies inside the
 // eager window the warp's lane 0 walks the codes at once and the side skips the executor.
 // A side still running after `budget` strips is handed to the block-per-side inspector (escalation).
-template <int R, bool FOLD>
+template <int R>
 __global__ void __launch_bounds__(WARPS * 32) k_inspect(DevParams P, Batch b, int4* ring, int rmask,
                                                          SideArrays sa, ExecPlan pl, int budget) {
     __shared__ SmemDP sm;
@@ -177,7 +185,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_inspect(DevParams P, Batch b, in
         if (side >= nsides) break;
         setup_side(b, side, io);
         SideOut o;
-        run_side<R, MODE_INSPECT, true, FOLD, false>(P, io, o);
+        run_side<R, MODE_INSPECT, true, false>(P, io, o);
         __syncwarp();  // eager corner codes (shared memory) written by lanes 0..4 -> read by lane 0
         if (lane == 0) {
             if (o.flags & SF_ESCALATE) {
@@ -199,7 +207,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_inspect(DevParams P, Batch b, in
 }
 
 // Block per side (long sides, escalated by k_inspect): the CTA's warps pipeline the side's strips.
-template <int R, bool FOLD>
+template <int R>
 __global__ void __launch_bounds__(WARPS * 32) k_inspect_block(DevParams P, Batch b, int4* ring, int rmask,
                                                                SideArrays sa, ExecPlan pl) {
     __shared__ SmemDP sm;
@@ -221,13 +229,13 @@ __global__ void __launch_bounds__(WARPS * 32) k_inspect_block(DevParams P, Batch
         io.ps = &ps;
         setup_side(b, side, io);
         SideOut o;
-        run_side<R, MODE_INSPECT, false, FOLD, true>(P, io, o);
+        run_side<R, MODE_INSPECT, false, true>(P, io, o);
         if (threadIdx.x == 0) write_side(P, sa, side, o, o.flags, 0ull, 0);
         __syncthreads();
     }
 }
 
-template <int R, bool FOLD>
+template <int R>
 __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int4* ring, int rmask,
                                                         long long* cells, int* counter) {
     __shared__ SmemDP sm;
@@ -243,7 +251,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int
         if (side >= nsides) break;
         setup_side(b, side, io);
         SideOut o;
-        run_side<R, MODE_CENSUS, false, FOLD, false>(P, io, o);
+        run_side<R, MODE_CENSUS, false, false>(P, io, o);
         if (lane == 0) cells[side] = (o.flags & SF_RING) ? -1 : o.cells;
         __syncwarp();
     }
@@ -253,7 +261,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int
 // Trimmed executor: the DP over [0,i*]x[0,j*] only, writing traceback codes.  Length binning
 // as a schedule: the CTAs first take the long sides (bins >= 3, block per side, strips pipelined
 // across the CTA's warps), then every warp takes short sides (bins 1-2, warp per side), larger bins first.
-template <int R, bool FOLD>
+template <int R>
 __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, int4* ring, int rmask,
                                                          SideArrays sa, ExecPlan pl, int lo, int hi, int nblock,
                                                          long long base, Outputs out) {
@@ -283,7 +291,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, in
         io.stab = out.stab + pl.soff[side];
         io.maxsw = sa.maxsw[side];
         SideOut o;
-        run_side<R, MODE_EXEC, false, FOLD, true>(P, io, o);
+        run_side<R, MODE_EXEC, false, true>(P, io, o);
         if (threadIdx.x == 0 && (o.flags & SF_RING)) atomicOr(&sa.flags[side], SF_RING);
         __syncthreads();
     }
@@ -303,7 +311,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, in
         io.codes = out.codes + (pl.woff[side] - base);
         io.stab = out.stab + pl.soff[side];
         SideOut o;
-        run_side<R, MODE_EXEC, false, FOLD, false>(P, io, o);
+        run_side<R, MODE_EXEC, false, false>(P, io, o);
         if (lane == 0 && (o.flags & SF_RING)) atomicOr(&sa.flags[side], SF_RING);
         __syncwarp();
     }
@@ -629,7 +637,7 @@ int pick_R() {  // read at fastz_create
 template <int R>
 static int bps_of() {
     int n = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_inspect<R, true>, WARPS * 32, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_inspect<R>, WARPS * 32, 0);
     return n > 0 ? n : 1;
 }
 
@@ -637,13 +645,8 @@ int inspector_blocks_per_sm(int R) { return R == 2 ? bps_of<2>() : bps_of<4>(); 
 
 #define FZ_DISPATCH(KERNEL, GRID, ...)                                                   \
     do {                                                                                 \
-        if (R == 2) {                                                                    \
-            if (P.fold_oe) KERNEL<2, true><<<GRID, WARPS * 32, 0, st>>>(__VA_ARGS__);    \
-            else KERNEL<2, false><<<GRID, WARPS * 32, 0, st>>>(__VA_ARGS__);             \
-        } else {                                                                         \
-            if (P.fold_oe) KERNEL<4, true><<<GRID, WARPS * 32, 0, st>>>(__VA_ARGS__);    \
-            else KERNEL<4, false><<<GRID, WARPS * 32, 0, st>>>(__VA_ARGS__);             \
-        }                                                                                \
+        if (R == 2) KERNEL<2><<<GRID, WARPS * 32, 0, st>>>(__VA_ARGS__);                 \
+        else KERNEL<4><<<GRID, WARPS * 32, 0, st>>>(__VA_ARGS__);                        \
     } while (0)
 
 // Inspector escalation of long sides to the block-per-side inspector (FASTZ_ESCALATE_STRIPS, strips; 0 = off).

@@ -49,7 +49,8 @@ constexpr int BLK = 32;
 constexpr int PIPE_SLOTS = 8;  // 2K slots for K = 4 warps: a slot is reused only after its consumer finished
 
 struct WarpSmem {
-    int2 cp[CP_RING + BLK]; // column profiles, ring over relative columns (+BLK mirrored)
+    int co[CP_RING + BLK];  // column codes of the query side as substitution-table byte offsets (code * SUBTAB_CODE),
+                            // ring over relative columns (+BLK mirrored)
     int4 bin[BLK];          // boundary row staging {X, D, W, -}: lane 0's input of the current block
     int4 bout[BLK];         // lane 31's bottom-row outputs {X, D, W, -} awaiting the global ring
 };
@@ -82,7 +83,7 @@ struct SideIO {
     int4* __restrict__ ring;            // boundary ring (per warp in SOLO, per CTA in PIPE), rmask + 1 entries
     int rmask;
     WarpSmem* ws;                       // shared staging of this warp
-    const int2* cptab;                  // shared: 5 profiles (query base 0..3, zero)
+    unsigned subtab;                    // shared address of the substitution table (dp.cuh, SUBTAB_*)
     uint8_t* ecodes;                    // shared: EAGER_W^2 eager codes (inspector)
     int eager_max;
     uint32_t* __restrict__ codes;       // executor: the side's code words
@@ -115,10 +116,10 @@ __device__ __forceinline__ int query_code(const SideIO& io, int c) {
 }
 
 __device__ __forceinline__ void cp_store(const SideIO& io, int rc, int code) {
-    const int2 v = io.cptab[code];
+    const int v = code * SUBTAB_CODE;
     const int idx = rc & (CP_RING - 1);
-    io.ws->cp[idx] = v;
-    if (idx < BLK) io.ws->cp[idx + CP_RING] = v;
+    io.ws->co[idx] = v;
+    if (idx < BLK) io.ws->co[idx + CP_RING] = v;
 }
 
 // Boundary row value at column c: the ring holds exact entries up to column lim, beyond it the row is dead
@@ -131,7 +132,7 @@ __device__ __forceinline__ int4 boundary(const int4* __restrict__ ring, int rmas
 
 __device__ __forceinline__ void pipe_wait() { __nanosleep(100); }
 
-template <int R, int MODE, bool EAGER, bool FOLD, bool PIPE>
+template <int R, int MODE, bool EAGER, bool PIPE>
 __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, SideOut& out) {
     constexpr int H = StripGeom<R>::H;
     constexpr int SPW = StripGeom<R>::SPW;
@@ -210,7 +211,9 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         const int top = s * H;
 
         // ------------------------------------------------------------------ strip set-up
-        int sel[R], X[R], I[R], W[R];
+        static_assert(R % 2 == 0, "rows per lane come in pairs (substitution table entries)");
+        unsigned tb[R / 2];  // per row pair: shared address of this lane's replica of the pair's table entries
+        int X[R], I[R], W[R];
         const int r0 = top + lane * R;
         int nvalid = M - r0 + 1;
         nvalid = nvalid < 0 ? 0 : (nvalid > R ? R : nvalid);
@@ -219,7 +222,8 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             const int r = r0 + k;
             int a = 0;
             if (r >= 1 && r <= M) a = base_at(io.Apk, io.Aoff + r - 1);
-            sel[k] = row_selector(a);
+            if (k % 2 == 0) tb[k / 2] = io.subtab + (unsigned)(a * 4 * SUBTAB_ENTRY) + (unsigned)((lane & 15) * 8);
+            else tb[k / 2] += (unsigned)(a * SUBTAB_ENTRY);
             X[k] = NEG;
             I[k] = NEG;
             W[k] = (r <= M) ? Wleft0 : BIG;
@@ -277,6 +281,10 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         uint32_t cw = 0;
         int lastlive_t = -1;  // last 4-step group end at which this lane had a live cell (termination)
         int cacc = NEG;       // max X of this lane over the current 4-step group
+        int Xp[R];            // inspector: X of the previous (even) step, peak-tested with the next step
+        bool vp = false;
+#pragma unroll
+        for (int k = 0; k < R; ++k) Xp[k] = NEG;
         int tfinal = 0;
         int bfirst = INT_MAX, blast = -1;  // bottom row's first/last live column (from the parked values)
         if constexpr (PIPE) lastlive = s == 0 ? -1 : INT_MAX;  // unknown until strip s-1 has finished
@@ -323,16 +331,16 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             int wu = __shfl_sync(FULL, bq.z, src);
             // lane 0 replaces what lane 31 sent with the boundary row for its column (relative column tt)
             ld_shared3_if(is0, sgi + 16u * (unsigned)j, xu, du, wu);
-            int cmv = NEG;
             if (valid) {
-                const int2 cp = ws->cp[cbase + u];
+                const int co = ws->co[cbase + u];
+                int vs[R];
+#pragma unroll
+                for (int p = 0; p < R / 2; ++p) ld_shared2(fma_add(co, one, (int)tb[p]), vs[2 * p], vs[2 * p + 1]);
                 int xd = xdiag;
                 xdiag = xu;
-                int cm = NEG;
 #pragma unroll
                 for (int k = 0; k < R; ++k) {
-                    const int h = FOLD ? fma_add(prmt(cp.x, cp.y, sel[k]), one, xd)
-                                       : xd + prmt(cp.x, cp.y, sel[k]) + OE;
+                    const int h = fma_add(vs[k], one, xd);  // X_diag + sub(a_i, b_j) + O + E
                     const int d = __viaddmax_s32(du, mE, xu);
                     const int iv = __viaddmax_s32(I[k], mE, X[k]);
                     const int sr = __vimax3_s32(h, d, iv);
@@ -358,26 +366,47 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                     xu = xn;
                     du = d;
                     wu = wn;
-                    cm = k == 0 ? xn : imax(cm, xn);
                 }
                 bq.x = xu;
                 bq.y = du;
                 bq.z = wu;
-                cacc = imax(cacc, cm);
-                cmv = cm;
+#pragma unroll
+                for (int k = 0; k < R; k += 2) cacc = __vimax3_s32(cacc, X[k], X[k + 1]);
             }
             if constexpr (MODE == MODE_INSPECT) {
-                // peak (reading R5): rare, warp-uniform slow path; ties -> smaller row (columns only grow)
-                if (__any_sync(FULL, cmv >= best)) {
-                    const int c = start + rc;
+                // peak (reading R5): tested every second step against the group maximum (a rare, warp-uniform
+                // slow path then scans both steps' cells in column order; ties -> smaller row, columns only grow).
+                // Re-scanning a cell is harmless: only a strictly better score or an equal one in a smaller row
+                // moves the peak.
+                const bool odd = (j & 1) != 0;
+                if (!odd) {
 #pragma unroll
-                    for (int k = 0; k < R; ++k) {
-                        const int r = r0 + k;
-                        const bool better = valid && (X[k] > best || (X[k] == best && r < bi));
-                        best = better ? X[k] : best;
-                        bi = better ? r : bi;
-                        bj = better ? c : bj;
-                        upd |= better;
+                    for (int k = 0; k < R; ++k) Xp[k] = X[k];
+                    vp = valid;
+                }
+                if (odd || (CHK && tt == tlast)) {
+                    if (__any_sync(FULL, cacc >= best)) {
+                        const int c = start + rc;
+                        if (odd) {
+#pragma unroll
+                            for (int k = 0; k < R; ++k) {
+                                const int r = r0 + k;
+                                const bool better = vp && (Xp[k] > best || (Xp[k] == best && r < bi));
+                                best = better ? Xp[k] : best;
+                                bi = better ? r : bi;
+                                bj = better ? c - 1 : bj;
+                                upd |= better;
+                            }
+                        }
+#pragma unroll
+                        for (int k = 0; k < R; ++k) {
+                            const int r = r0 + k;
+                            const bool better = valid && (X[k] > best || (X[k] == best && r < bi));
+                            best = better ? X[k] : best;
+                            bi = better ? r : bi;
+                            bj = better ? c : bj;
+                            upd |= better;
+                        }
                     }
                 }
             }
