@@ -173,6 +173,49 @@ typedef struct {
 } fastz_stats;
 int fastz_get_stats(fastz_ctx *c, fastz_stats *s);
 
+/*
+ * Seeding + ungapped filter (the stage before the gapped extension).  PAPER.md P:93:
+ * "a lightweight exact-match search identifies short sequences (19 base pairs long) to serve as seed sites
+ * ... the second stage filters the seed sites to obtain a shorter list of promising seed sites ... the third
+ * stage extends the filtered seed sites".  The paper fixes only the 19-bp span; the defaults are LASTZ's
+ * [ext] and the exact semantics are readings S1-S6 of DESIGN.md:
+ *   pattern     spaced seed over '0'/'1', NUL-terminated, span 1..32, 1..16 care positions ('1'), first and
+ *               last character '1'; default "1110100110010101111" (12of19).  A hit (t, q) needs the target
+ *               and query words (bases at the care positions) to be equal -- S1/S2.
+ *   transitions 1: additionally allow one transition (A<->G, C<->T) at one care position (default 1) -- S2.
+ *   xdrop       X >= 0 of the ungapped x-drop walk right of and left of each hit along its diagonal; a walk
+ *               stops when its running score falls more than X below its maximum (default 910) -- S3.
+ *   hspthresh   an HSP (the two walks' best extents) is kept iff its score >= hspthresh (default 3000) -- S4.
+ * Scores use the context's sub[] matrix.
+ */
+typedef struct {
+    char pattern[64];
+    int32_t transitions;
+    int32_t xdrop;
+    int32_t hspthresh;
+    int32_t reserved;
+} fastz_seed_params;
+
+/* An HSP: the ungapped segment T[t_start, t_start+length) x Q[q_start, q_start+length) and its score. */
+typedef struct {
+    int64_t t_start, q_start;
+    int32_t length, score;
+} fastz_hsp;
+
+void fastz_default_seed_params(fastz_seed_params *sp);
+
+/*
+ * Find the HSPs between the context's target and query (forward strands) on the device: spaced-seed hits,
+ * ungapped x-drop filter, identical HSPs reported once (S5), sorted by anchor (S6).  `hsps` (may be NULL)
+ * receives the HSPs and `anchors` (may be NULL) their cut points for fastz_extend_seeds: the HSP midpoint
+ * (t_start + length/2, q_start + length/2).  Both are host buffers of `cap` entries; if cap is too small,
+ * nothing is copied, *n_out holds the required count and FASTZ_ETRUNC is returned.  *n_hits (may be NULL)
+ * receives the number of raw seed hits.  Synchronizes the stream.  Errors: EINVAL (bad pattern/params),
+ * ERANGE (a single query word with more hits than device memory holds), ENOMEM, ECUDA.
+ */
+int fastz_find_hsps(fastz_ctx *c, const fastz_seed_params *sp, fastz_hsp *hsps, fastz_seed *anchors, int64_t cap,
+                    int64_t *n_out, int64_t *n_hits);
+
 /* Release everything; NULL-safe. */
 void fastz_destroy(fastz_ctx *c);
 

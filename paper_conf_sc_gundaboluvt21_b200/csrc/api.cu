@@ -10,6 +10,7 @@
 #include <algorithm>
 #include <climits>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -54,6 +55,9 @@ struct fastz_ctx {
     DBuf seeds, score, ti, qj, flags, eops, bound, maxsw, esc, nstrip;
     DBuf woff, soff, roff, bin, list, counters, totals, tmpa, tmpb, tmpc, scan_tmp, wl, wlo;
     DBuf codes, stab, runs, nruns, ciglen, cigar, recs, cells, ring, small;
+    // seeding (fastz_find_hsps)
+    DBuf s_kin, s_kout, s_pin, s_pout, s_start, s_cnt, s_off, s_hits, s_hsp, s_keep, s_sel, s_list, s_list2,
+        s_k1, s_k2, s_i1, s_i2, s_flag, s_pos, s_out, s_anch, s_tmp;
     int R = 4, grid = 0, nslots = 0, rmask = 0;
     int64_t n = 0, cigar_bytes = 0, nexec = 0;
     int nwaves = 0;
@@ -240,6 +244,14 @@ void fastz_default_params(fastz_params* p) {
     p->eager_max = 16;
 }
 
+void fastz_default_seed_params(fastz_seed_params* sp) {
+    memset(sp, 0, sizeof(*sp));
+    strcpy(sp->pattern, "1110100110010101111");  // 12of19 (LASTZ default [ext]; 19-bp seeds)
+    sp->transitions = 1;
+    sp->xdrop = 910;
+    sp->hspthresh = 3000;
+}
+
 const char* fastz_strerror(int status) {
     static thread_local std::string s;
     const char* base = "unknown status";
@@ -266,7 +278,9 @@ void fastz_destroy(fastz_ctx* c) {
                     &c->flags, &c->eops, &c->bound, &c->maxsw, &c->esc, &c->nstrip, &c->woff, &c->soff, &c->roff, &c->bin, &c->list,
                     &c->counters, &c->totals, &c->tmpa, &c->tmpb, &c->tmpc, &c->scan_tmp, &c->wl, &c->wlo, &c->codes,
                     &c->stab, &c->runs, &c->nruns, &c->ciglen, &c->cigar, &c->recs, &c->cells, &c->ring,
-                    &c->small};
+                    &c->small, &c->s_kin, &c->s_kout, &c->s_pin, &c->s_pout, &c->s_start, &c->s_cnt, &c->s_off,
+                    &c->s_hits, &c->s_hsp, &c->s_keep, &c->s_sel, &c->s_list, &c->s_list2, &c->s_k1, &c->s_k2,
+                    &c->s_i1, &c->s_i2, &c->s_flag, &c->s_pos, &c->s_out, &c->s_anch, &c->s_tmp};
     for (DBuf* b : bufs) dfree(c, *b);
     if (c->ev_ok)
         for (auto& e : c->ev) cudaEventDestroy(e);
@@ -576,6 +590,137 @@ int fastz_get_stats(fastz_ctx* c, fastz_stats* s) {
 int fastz_int_peak(int device, float ms, double* ops_per_s, double* sm_clock_mhz) {
     if (!ops_per_s || !sm_clock_mhz) return fail(FASTZ_EINVAL, "NULL argument");
     CK(int_peak_run(device, ms, ops_per_s, sm_clock_mhz));
+    return 0;
+}
+
+static_assert(sizeof(HspOut) == sizeof(fastz_hsp), "fastz_hsp layout");
+
+int fastz_find_hsps(fastz_ctx* c, const fastz_seed_params* spp, fastz_hsp* hsps, fastz_seed* anchors, int64_t cap,
+                    int64_t* n_out, int64_t* n_hits) {
+    if (!c || !spp || !n_out) return fail(FASTZ_EINVAL, "NULL argument");
+    if (cap < 0) return fail(FASTZ_EINVAL, "cap < 0");
+    // S1: parse the spaced seed
+    SeedPattern sp{};
+    const size_t L = strnlen(spp->pattern, sizeof(spp->pattern));
+    if (L == 0 || L > 32) return fail(FASTZ_EINVAL, "seed pattern span must be 1..32");
+    for (size_t i = 0; i < L; ++i) {
+        if (spp->pattern[i] == '1') {
+            if (sp.w == 16) return fail(FASTZ_EINVAL, "seed pattern has more than 16 care positions");
+            sp.off[sp.w++] = (int)i;
+        } else if (spp->pattern[i] != '0') {
+            return fail(FASTZ_EINVAL, "seed pattern characters must be '0' or '1'");
+        }
+    }
+    if (spp->pattern[0] != '1' || spp->pattern[L - 1] != '1')
+        return fail(FASTZ_EINVAL, "seed pattern must start and end with '1'");
+    if (spp->xdrop < 0) return fail(FASTZ_EINVAL, "xdrop must be >= 0");
+    sp.L = (int)L;
+    UngappedParams up{};
+    for (int k = 0; k < 16; ++k) up.sub[k] = c->prm.sub[k];
+    up.xdrop = spp->xdrop;
+    up.hspthresh = spp->hspthresh;
+    const int nvar = spp->transitions ? 1 + sp.w : 1;
+    CK(cudaSetDevice(c->device));
+    cudaStream_t st = c->stream;
+    const long long nt = c->tlen >= sp.L ? (long long)c->tlen - sp.L + 1 : 0;
+    const long long nq = c->qlen >= sp.L ? (long long)c->qlen - sp.L + 1 : 0;
+    const long long nkeys = 1LL << (2 * sp.w);
+    const bool dense = sp.w <= 12;
+    long long HIT_CAP = 1LL << 25;  // hits per query chunk (24 B of scratch each); env override for tests
+    if (const char* e = getenv("FASTZ_SEED_HIT_CAP")) HIT_CAP = std::max(1LL, atoll(e));
+    long long QC = std::min<long long>(std::max<long long>(nq, 1), std::min(1LL << 22, HIT_CAP));
+
+    // index of the target: (word, position) sorted, dense bucket starts
+    const size_t tmpb = seed_sort_tmp_bytes(std::max(std::max(nt, HIT_CAP), QC + 1));
+    AL(s_tmp, tmpb);
+    AL(s_kin, 4 * (nt + 1));
+    AL(s_kout, 4 * (nt + 1));
+    AL(s_pin, 4 * (nt + 1));
+    AL(s_pout, 4 * (nt + 1));
+    if (dense) AL(s_start, 4 * (nkeys + 1));
+    AL(s_cnt, 8 * (QC + 1));
+    AL(s_off, 8 * (QC + 1));
+    CK(seed_keys(P_<uint32_t>(c->Tf), nt, sp, P_<uint32_t>(c->s_kin), P_<int>(c->s_pin), st));
+    CK(seed_sort_words(c->s_tmp.p, tmpb, P_<uint32_t>(c->s_kin), P_<uint32_t>(c->s_kout), P_<int>(c->s_pin),
+                       P_<int>(c->s_pout), nt, 2 * sp.w, st));
+    const int* start = nullptr;
+    if (dense) {
+        CK(seed_bucket_start(P_<uint32_t>(c->s_kout), nt, P_<int>(c->s_start), nkeys, st));
+        start = P_<int>(c->s_start);
+    }
+    // query chunks: count -> scan -> (D2H total) -> write hits -> ungapped walks -> select survivors
+    long long q0 = 0, hits_total = 0, nlist = 0, list_cap = 0;
+    while (q0 < nq) {
+        const long long nqc = std::min(QC, nq - q0);
+        CK(seed_count(P_<uint32_t>(c->Qf), q0, nqc, sp, nvar, P_<uint32_t>(c->s_kout), P_<int>(c->s_pout), start, nt,
+                      P_<long long>(c->s_cnt), P_<long long>(c->s_off), c->s_tmp.p, tmpb, st));
+        long long nh = 0;
+        CK(cudaMemcpyAsync(&nh, P_<long long>(c->s_off) + nqc, sizeof(nh), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        if (nh > HIT_CAP && nqc > 1) {  // too many hits for the scratch: halve the chunk
+            QC = std::max<long long>(1, nqc / 2);
+            continue;
+        }
+        if (nh > (1LL << 31) - 1) return fail(FASTZ_ERANGE, "a query word has more than 2^31 seed hits");
+        if (nh > 0) {
+            AL(s_hits, 8 * nh);
+            AL(s_hsp, 16 * nh);
+            AL(s_keep, nh);
+            AL(s_sel, 16 * nh + 16);
+            const size_t tb2 = seed_sort_tmp_bytes(nh);
+            if (tb2 > c->s_tmp.cap) AL(s_tmp, tb2);
+            CK(seed_write_extend(P_<uint32_t>(c->Tf), P_<uint32_t>(c->Qf), c->tlen, c->qlen, q0, nqc, sp, nvar,
+                                 P_<uint32_t>(c->s_kout), P_<int>(c->s_pout), start, nt, P_<long long>(c->s_off), nh,
+                                 P_<int2>(c->s_hits), up, P_<int4>(c->s_hsp), P_<unsigned char>(c->s_keep), st));
+            int* nsel_d = reinterpret_cast<int*>(P_<int4>(c->s_sel) + nh);
+            CK(seed_select(c->s_tmp.p, c->s_tmp.cap, P_<int4>(c->s_hsp), P_<unsigned char>(c->s_keep), nh,
+                           P_<int4>(c->s_sel), nsel_d, st));
+            int nsel = 0;
+            CK(cudaMemcpyAsync(&nsel, nsel_d, sizeof(int), cudaMemcpyDeviceToHost, st));
+            CK(cudaStreamSynchronize(st));
+            if (nsel > 0) {
+                if (nlist + nsel > list_cap) {  // grow the HSP list, keeping its contents
+                    list_cap = std::max<long long>(2 * list_cap, nlist + nsel);
+                    AL(s_list2, 16 * list_cap);
+                    if (nlist) CK(cudaMemcpyAsync(c->s_list2.p, c->s_list.p, 16 * nlist, cudaMemcpyDeviceToDevice, st));
+                    std::swap(c->s_list, c->s_list2);
+                }
+                CK(cudaMemcpyAsync(P_<int4>(c->s_list) + nlist, c->s_sel.p, 16 * (size_t)nsel,
+                                   cudaMemcpyDeviceToDevice, st));
+                nlist += nsel;
+            }
+        }
+        hits_total += nh;
+        q0 += nqc;
+    }
+    if (n_hits) *n_hits = hits_total;
+    long long nu = 0;
+    if (nlist > 0) {
+        AL(s_k1, 8 * nlist);
+        AL(s_k2, 16 * nlist);
+        AL(s_i1, 4 * nlist);
+        AL(s_i2, 4 * nlist);
+        AL(s_flag, 4 * (nlist + 1));
+        AL(s_pos, 4 * (nlist + 1));
+        const size_t tb3 = seed_sort_tmp_bytes(nlist);
+        if (tb3 > c->s_tmp.cap) AL(s_tmp, tb3);
+        CK(seed_finish_sort(c->s_tmp.p, c->s_tmp.cap, P_<int4>(c->s_list), nlist, P_<unsigned long long>(c->s_k1),
+                            P_<unsigned long long>(c->s_k2), P_<int>(c->s_i1), P_<int>(c->s_i2), st));
+        AL(s_out, sizeof(HspOut) * nlist);
+        AL(s_anch, 16 * nlist);
+        CK(seed_unique_emit(c->s_tmp.p, c->s_tmp.cap, P_<int4>(c->s_list), P_<int>(c->s_i1), nlist, P_<int>(c->s_flag),
+                            P_<int>(c->s_pos), P_<HspOut>(c->s_out), P_<long long>(c->s_anch), st));
+        int nuu = 0;
+        CK(cudaMemcpyAsync(&nuu, P_<int>(c->s_pos) + nlist, sizeof(int), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        nu = nuu;
+    }
+    *n_out = nu;
+    if (nu > cap) return fail(FASTZ_ETRUNC, "HSP buffer too small: " + std::to_string(nu) + " needed");
+    if (nu > 0 && hsps) CK(cudaMemcpyAsync(hsps, c->s_out.p, sizeof(fastz_hsp) * nu, cudaMemcpyDeviceToHost, st));
+    if (nu > 0 && anchors)
+        CK(cudaMemcpyAsync(anchors, c->s_anch.p, sizeof(fastz_seed) * nu, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
     return 0;
 }
 

@@ -85,4 +85,39 @@ cudaError_t launch_combine_write(const DevParams& P, const Batch& b, const SideA
                                  const ExecPlan& pl, const Outputs& o, cudaStream_t st);
 cudaError_t int_peak_run(int device, float ms, double* ops_per_s, double* mhz);
 
+
+// ---------------------------------------------------------------------------------------- seeding (seeds.cu)
+struct SeedPattern {
+    int L, w;      // span, care positions (1..16)
+    int off[16];   // care offsets, ascending
+};
+struct UngappedParams {
+    int sub[16];   // sub[4a+b], a = target base, b = query base
+    int xdrop, hspthresh;
+};
+struct HspOut {    // layout of fastz_hsp
+    long long t_start, q_start;
+    int length, score;
+};
+size_t seed_sort_tmp_bytes(long long n);
+cudaError_t seed_keys(const uint32_t* Tf, long long nt, const SeedPattern& sp, uint32_t* keys, int* pos,
+                      cudaStream_t st);
+cudaError_t seed_sort_words(void* tmp, size_t tmp_bytes, const uint32_t* kin, uint32_t* kout, const int* vin,
+                            int* vout, long long n, int bits, cudaStream_t st);
+cudaError_t seed_bucket_start(const uint32_t* skeys, long long nt, int* start, long long nkeys, cudaStream_t st);
+cudaError_t seed_count(const uint32_t* Qf, long long q0, long long nq, const SeedPattern& sp, int nvar,
+                       const uint32_t* skeys, const int* spos, const int* start, long long nt, long long* cnt,
+                       long long* off, void* tmp, size_t tmp_bytes, cudaStream_t st);
+cudaError_t seed_write_extend(const uint32_t* Tf, const uint32_t* Qf, int tlen, int qlen, long long q0, long long nq,
+                              const SeedPattern& sp, int nvar, const uint32_t* skeys, const int* spos,
+                              const int* start, long long nt, const long long* off, long long nh, int2* hits,
+                              const UngappedParams& up, int4* hsp, unsigned char* keep, cudaStream_t st);
+cudaError_t seed_select(void* tmp, size_t tmp_bytes, const int4* hsp, const unsigned char* keep, long long nh,
+                        int4* out, int* nsel, cudaStream_t st);
+// k1: n keys, k2: 2n keys, i1/i2: n ints; the final order is left in i1
+cudaError_t seed_finish_sort(void* tmp, size_t tmp_bytes, const int4* hs, long long n, unsigned long long* k1,
+                             unsigned long long* k2, int* i1, int* i2, cudaStream_t st);
+cudaError_t seed_unique_emit(void* tmp, size_t tmp_bytes, const int4* hs, const int* order, long long n, int* flag,
+                             int* pos, HspOut* out, long long* anchors, cudaStream_t st);
+
 }  // namespace fz

@@ -162,13 +162,16 @@ __device__ __forceinline__ void write_side(const DevParams& P, const SideArrays&
     sa.nstrip[side] = notrim ? o.nstrips : -1;
 }
 
+#ifndef INSPECT_MIN_BLOCKS
+#define INSPECT_MIN_BLOCKS 1  // resident CTAs per SM the register allocation must allow (occupancy)
+#endif
 // ------------------------------------------------------------------------------------------------- inspector
 // Persistent: each warp pops one-sided extensions from an atomic queue (load balance replaces the paper's
 // 32 CUDA streams).  Score-only DP + eager 17x17 corner codes; when the peak lies inside the
 // eager window the warp's lane 0 walks the codes at once and the side skips the executor.
 // A side still running after `budget` strips is handed to the block-per-side inspector (escalation).
 template <int R>
-__global__ void __launch_bounds__(WARPS * 32) k_inspect(DevParams P, Batch b, int4* ring, int rmask,
+__global__ void __launch_bounds__(WARPS * 32, INSPECT_MIN_BLOCKS) k_inspect(DevParams P, Batch b, int4* ring, int rmask,
                                                          SideArrays sa, ExecPlan pl, int budget) {
     __shared__ SmemDP sm;
     smem_init(sm, P);

@@ -41,7 +41,10 @@ namespace fz {
 enum { MODE_INSPECT = 0, MODE_EXEC = 1, MODE_CENSUS = 2 };
 
 #ifndef STEADY_UNROLL
-#define STEADY_UNROLL 4  // steps per unrolled steady-state body (4 or 8; 16 overflows the I-cache)
+#define STEADY_UNROLL 8  // steps per unrolled steady-state body (8: one termination test per body; 16 overflows the I-cache)
+#endif
+#ifndef TERM_MASK
+#define TERM_MASK 7  // termination test every TERM_MASK + 1 steps (u & TERM_MASK == TERM_MASK; t is a multiple of 8)
 #endif
 // steps per staging block (refill of boundary/profiles, park of the bottom row): BLK for SOLO; PIPE uses 16 so a
 // consumer strip trails its producer by fewer columns (flush granularity + prefetch distance)
@@ -141,7 +144,7 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
     const bool stager = BK == 32 || lane < BK;  // lanes that move one staging entry per block
     const int src = (lane + 31) & 31;
     const int M = io.M, N = io.N;
-    const int E = P.E, OE = P.OE, OEmY = P.OE - P.Y, mE = -P.E, mOE = -P.OE;
+    const int E = P.E, OE = P.OE, mY = -P.Y, mE = -P.E, mOE = -P.OE;
     const int one = P.one, zero = P.zero;
     const int rmask = io.rmask;
     int4* __restrict__ ring = io.ring;
@@ -344,9 +347,12 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                     const int d = __viaddmax_s32(du, mE, xu);
                     const int iv = __viaddmax_s32(I[k], mE, X[k]);
                     const int sr = __vimax3_s32(h, d, iv);
-                    const int thr = imax(wu, W[k]);
-                    const int xn = kill_fma(sr, thr, mOE, one, zero);
-                    const int wn = __viaddmax_s32(xn, OEmY, thr);
+                    // W = max(thr, S_raw - Y) with thr = max(W_up, W_left): for a dead cell S_raw - Y < thr, so
+                    // this equals max(thr, S_live - Y) (reading R3), and since Y >= 0 the cell is live iff
+                    // S_raw >= W (S >= thr => W <= S; S < thr => W >= thr > S): the threshold max and the
+                    // live test share one VIMNMX3, S - Y runs on the FMA pipe
+                    const int wn = __vimax3_s32(wu, W[k], fma_add(sr, one, mY));
+                    const int xn = kill_fma(sr, wn, mOE, one, zero);
                     if constexpr (MODE == MODE_EXEC) {
                         const uint32_t code = cell_code(h, d, iv, du, xu, I[k], X[k], E);
                         cw |= code << ((((j % SPW) * R) + k) * 4);
@@ -423,7 +429,7 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                 lastlive_t = imax(lastlive_t, __viaddmin_s32(cacc, -NEG - 1, tt));
                 cacc = NEG;
             }
-            if (j == 3 && tt >= 31) {
+            if (j == 3 && (u & TERM_MASK) == TERM_MASK && tt >= 31) {
                 // done at lane 31's column x = start + tt - 31 iff every lane has been dead since it processed
                 // x (step tt - 31 + lane) and the boundary row has no live cell at or after x
                 const unsigned bal = __ballot_sync(FULL, lastlive_t < tt - 31 + lane);

@@ -25,7 +25,7 @@ OPT_NO_EAGER, OPT_NO_TRIM, OPT_NO_BINNING, OPT_NO_BLOCK, OPT_TRACEBACK_ABOVE_K =
 # names declared in include/fastz.h (checked by tests/test_abi.py against the header)
 EXPORTS = ["fastz_default_params", "fastz_create", "fastz_extend_seeds", "fastz_get_alignments",
            "fastz_get_alignments_device", "fastz_get_sides", "fastz_census", "fastz_get_stats",
-           "fastz_destroy", "fastz_strerror", "fastz_int_peak"]
+           "fastz_destroy", "fastz_strerror", "fastz_int_peak", "fastz_default_seed_params", "fastz_find_hsps"]
 
 
 class FastzError(RuntimeError):
@@ -50,6 +50,14 @@ class fastz_stats(ctypes.Structure):
                 ("bin_counts", ctypes.c_int64 * 8), ("exec_words", ctypes.c_int64), ("cigar_bytes", ctypes.c_int64),
                 ("n_launches", ctypes.c_int64), ("n_waves", ctypes.c_int64), ("n_escalated", ctypes.c_int64)]
 
+
+class fastz_seed_params(ctypes.Structure):
+    _fields_ = [("pattern", ctypes.c_char * 64), ("transitions", ctypes.c_int32), ("xdrop", ctypes.c_int32),
+                ("hspthresh", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+
+
+HSP_DTYPE = np.dtype([("t_start", "<i8"), ("q_start", "<i8"), ("length", "<i4"), ("score", "<i4")])
+assert HSP_DTYPE.itemsize == 24
 
 ALIGN_DTYPE = np.dtype([("score", "<i4"), ("left_score", "<i4"), ("right_score", "<i4"), ("flags", "<u4"),
                         ("t_start", "<i8"), ("t_end", "<i8"), ("q_start", "<i8"), ("q_end", "<i8"),
@@ -84,7 +92,11 @@ def lib() -> ctypes.CDLL:
     L.fastz_strerror.argtypes = [i32]
     L.fastz_strerror.restype = ctypes.c_char_p
     L.fastz_int_peak.argtypes = [i32, ctypes.c_float, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)]
-    for name in ("fastz_create", "fastz_extend_seeds", "fastz_get_alignments", "fastz_get_alignments_device",
+    L.fastz_default_seed_params.argtypes = [ctypes.POINTER(fastz_seed_params)]
+    L.fastz_default_seed_params.restype = None
+    L.fastz_find_hsps.argtypes = [vp, ctypes.POINTER(fastz_seed_params), vp, vp, i64, ctypes.POINTER(i64),
+                                  ctypes.POINTER(i64)]
+    for name in ("fastz_find_hsps", "fastz_create", "fastz_extend_seeds", "fastz_get_alignments", "fastz_get_alignments_device",
                  "fastz_get_sides", "fastz_census", "fastz_get_stats", "fastz_int_peak"):
         getattr(L, name).restype = i32
     _lib = L
@@ -192,6 +204,30 @@ def fastz_destroy(ctx: int):
         lib().fastz_destroy(ctx)
 
 
+def fastz_default_seed_params(**overrides) -> fastz_seed_params:
+    sp = fastz_seed_params()
+    lib().fastz_default_seed_params(ctypes.byref(sp))
+    for k, v in overrides.items():
+        setattr(sp, k, v.encode() if k == "pattern" else int(v))
+    return sp
+
+
+def fastz_find_hsps(ctx: int, sp: fastz_seed_params | None = None):
+    """(HSPs as a HSP_DTYPE array in anchor order, anchors as an (n, 2) int64 array, raw hit count)."""
+    sp = sp if sp is not None else fastz_default_seed_params()
+    n, hits = ctypes.c_int64(0), ctypes.c_int64(0)
+    st = lib().fastz_find_hsps(ctx, ctypes.byref(sp), None, None, 0, ctypes.byref(n), ctypes.byref(hits))
+    if st not in (FASTZ_OK, FASTZ_ETRUNC):
+        _check(st)
+    cap = int(n.value)
+    hs = np.zeros(cap, dtype=HSP_DTYPE)
+    an = np.zeros((cap, 2), dtype=np.int64)
+    if cap:
+        _check(lib().fastz_find_hsps(ctx, ctypes.byref(sp), hs.ctypes.data, an.ctypes.data, cap, ctypes.byref(n),
+                                     ctypes.byref(hits)))
+    return hs, an, int(hits.value)
+
+
 def fastz_int_peak(device: int = 0, ms: float = 200.0):
     ops, mhz = ctypes.c_double(), ctypes.c_double()
     _check(lib().fastz_int_peak(device, ms, ctypes.byref(ops), ctypes.byref(mhz)))
@@ -242,6 +278,10 @@ class Aligner:
 
     def sides(self):
         return fastz_get_sides(self.ctx, self.n)
+
+    def find_hsps(self, **seed_params):
+        """Seeding + ungapped filter on this context's sequences (NEXT-4): (hsps, anchors, hits)."""
+        return fastz_find_hsps(self.ctx, fastz_default_seed_params(**seed_params))
 
     def census(self) -> np.ndarray:
         return fastz_census(self.ctx, self.n)
