@@ -237,7 +237,7 @@ def run_fastz(args, ws, rank, local):
             dist.barrier()
         t0 = time.perf_counter()
         al.extend_only(seeds_h)
-        res = al.results()
+        res = al.results_pinned()
         e2e_t.append(time.perf_counter() - t0)
         d2h = res.rec.nbytes + len(res.cigar)
     e2e_ms = sum(e2e_t) / len(e2e_t) * 1e3

@@ -81,6 +81,10 @@ typedef struct {
 #define FASTZ_OPT_NO_BINNING 4   /* one executor queue, warp per side, no length order (P:209-211 off) */
 #define FASTZ_OPT_NO_BLOCK 8     /* no block-per-side scheduling of long sides (inspector and executor) */
 #define FASTZ_OPT_TRACEBACK_ABOVE_K 16 /* traceback only seeds with score >= K; others get an empty CIGAR */
+#define FASTZ_OPT_QUERY_REVCOMP 32 /* the context's query is the reverse complement of the `query` passed to
+                                      fastz_create (minus strand, NEXT-4): seeds, HSPs and alignments use
+                                      reverse-complement query coordinates; an invalid character is reported at
+                                      its index in the caller's string */
 
 /* A seed is a cut point: the right extension starts at T[tpos], Q[qpos]; the left one at T[tpos-1],
  * Q[qpos-1] going backwards.  0 <= tpos <= tlen, 0 <= qpos <= qlen. */

@@ -134,7 +134,7 @@ int check_params(const fastz_params* p) {
     return 0;
 }
 
-int upload_seq(fastz_ctx* c, const char* src, int64_t len, DBuf& fwd, DBuf& rev, int64_t base_index) {
+int upload_seq(fastz_ctx* c, const char* src, int64_t len, DBuf& fwd, DBuf& rev, int64_t base_index, int revcomp) {
     const size_t words = (size_t)((len + 15) / 16) + 4;
     int r;
     if ((r = dalloc(c, fwd, words * 4))) return r;
@@ -151,7 +151,7 @@ int upload_seq(fastz_ctx* c, const char* src, int64_t len, DBuf& fwd, DBuf& rev,
     if ((r = dalloc(c, c->small, 64))) return r;
     long long init = LLONG_MAX;
     CK(cudaMemcpyAsync(c->small.p, &init, sizeof(init), cudaMemcpyHostToDevice, c->stream));
-    CK(launch_pack(dsrc, len, P_<uint32_t>(fwd), P_<uint32_t>(rev), P_<long long>(c->small), c->stream));
+    CK(launch_pack(dsrc, len, P_<uint32_t>(fwd), P_<uint32_t>(rev), P_<long long>(c->small), revcomp, c->stream));
     long long bad = 0;
     CK(cudaMemcpyAsync(&bad, c->small.p, sizeof(bad), cudaMemcpyDeviceToHost, c->stream));
     CK(cudaStreamSynchronize(c->stream));
@@ -330,7 +330,8 @@ int fastz_create(const fastz_params* p, const char* target, int64_t tlen, const 
     c->dp.eager_max = p->eager_max;
     c->tlen = (int)tlen;
     c->qlen = (int)qlen;
-    if ((r = upload_seq(c, target, tlen, c->Tf, c->Tr, 0)) || (r = upload_seq(c, query, qlen, c->Qf, c->Qr, tlen))) {
+    if ((r = upload_seq(c, target, tlen, c->Tf, c->Tr, 0, 0)) ||
+        (r = upload_seq(c, query, qlen, c->Qf, c->Qr, tlen, (p->options & FASTZ_OPT_QUERY_REVCOMP) ? 1 : 0))) {
         fastz_destroy(c);
         return r;
     }

@@ -56,7 +56,7 @@ struct Outputs {
 
 int pick_R();  // rows per lane (FASTZ_R env: 2, 4 or 8; default 4)
 
-cudaError_t launch_pack(const char* src, int64_t n, uint32_t* fwd, uint32_t* rev, long long* bad,
+cudaError_t launch_pack(const char* src, int64_t n, uint32_t* fwd, uint32_t* rev, long long* bad, int revcomp,
                         cudaStream_t st);
 cudaError_t launch_validate_seeds(const long long* seeds, int n, int tlen, int qlen, long long* bad,
                                   cudaStream_t st);

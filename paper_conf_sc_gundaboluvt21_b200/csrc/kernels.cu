@@ -22,32 +22,36 @@ __device__ __forceinline__ int code_of(unsigned char c) {
 }
 
 __global__ void k_pack(const char* __restrict__ src, long long n, uint32_t* __restrict__ fwd,
-                       uint32_t* __restrict__ rev, long long* bad) {
+                       uint32_t* __restrict__ rev, long long* bad, int revcomp) {
     const long long w = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     const long long nw = (n + 15) / 16;
     if (w >= nw) return;
+    // revcomp: the sequence is the reverse complement of src (A<->T, C<->G: code xor 3), so its forward copy
+    // reads src backwards and its reversed copy reads src forwards, both complemented
+    const uint32_t cx = revcomp ? 3u : 0u;
     uint32_t f = 0, r = 0;
 #pragma unroll 4
     for (int i = 0; i < 16; ++i) {
         const long long p = 16 * w + i;
         if (p < n) {
-            int c = code_of((unsigned char)src[p]);
-            if (c < 0) { atomicMin(bad, p); c = 0; }
-            f |= (uint32_t)c << (2 * i);
-            int cr = code_of((unsigned char)src[n - 1 - p]);
+            const long long pf = revcomp ? n - 1 - p : p;
+            int c = code_of((unsigned char)src[pf]);
+            if (c < 0) { atomicMin(bad, pf); c = 0; }
+            f |= ((uint32_t)c ^ cx) << (2 * i);
+            int cr = code_of((unsigned char)src[revcomp ? p : n - 1 - p]);
             if (cr < 0) cr = 0;
-            r |= (uint32_t)cr << (2 * i);
+            r |= ((uint32_t)cr ^ cx) << (2 * i);
         }
     }
     fwd[w] = f;
     rev[w] = r;
 }
 
-cudaError_t launch_pack(const char* src, int64_t n, uint32_t* fwd, uint32_t* rev, long long* bad,
+cudaError_t launch_pack(const char* src, int64_t n, uint32_t* fwd, uint32_t* rev, long long* bad, int revcomp,
                         cudaStream_t st) {
     const long long nw = (n + 15) / 16;
     if (nw == 0) return cudaSuccess;
-    k_pack<<<(unsigned)((nw + 255) / 256), 256, 0, st>>>(src, n, fwd, rev, bad);
+    k_pack<<<(unsigned)((nw + 255) / 256), 256, 0, st>>>(src, n, fwd, rev, bad, revcomp);
     return cudaGetLastError();
 }
 
@@ -162,8 +166,13 @@ __device__ __forceinline__ void write_side(const DevParams& P, const SideArrays&
     sa.nstrip[side] = notrim ? o.nstrips : -1;
 }
 
-#ifndef INSPECT_MIN_BLOCKS
-#define INSPECT_MIN_BLOCKS 1  // resident CTAs per SM the register allocation must allow (occupancy)
+// register budget of the inspector: by default only the CTA size is declared (ptxas then lands at 72
+// registers = 7 CTAs per SM, measured fastest); -DINSPECT_MIN_BLOCKS=n forces n resident CTAs per SM.  (An
+// explicit minimum of 1 is NOT the same: ptxas then spends 122 registers and occupancy drops to 4 CTAs.)
+#ifdef INSPECT_MIN_BLOCKS
+#define INSPECT_BOUNDS __launch_bounds__(WARPS * 32, INSPECT_MIN_BLOCKS)
+#else
+#define INSPECT_BOUNDS __launch_bounds__(WARPS * 32)
 #endif
 // ------------------------------------------------------------------------------------------------- inspector
 // Persistent: each warp pops one-sided extensions from an atomic queue (load balance replaces the paper's
@@ -171,7 +180,7 @@ __device__ __forceinline__ void write_side(const DevParams& P, const SideArrays&
 // eager window the warp's lane 0 walks the codes at once and the side skips the executor.
 // A side still running after `budget` strips is handed to the block-per-side inspector (escalation).
 template <int R>
-__global__ void __launch_bounds__(WARPS * 32, INSPECT_MIN_BLOCKS) k_inspect(DevParams P, Batch b, int4* ring, int rmask,
+__global__ void INSPECT_BOUNDS k_inspect(DevParams P, Batch b, int4* ring, int rmask,
                                                          SideArrays sa, ExecPlan pl, int budget) {
     __shared__ SmemDP sm;
     smem_init(sm, P);

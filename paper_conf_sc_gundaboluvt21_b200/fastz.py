@@ -170,7 +170,7 @@ def fastz_get_alignments(ctx: int):
     st = lib().fastz_get_alignments(ctx, None, 0, None, 0, ctypes.byref(n), ctypes.byref(nb))
     if st not in (FASTZ_OK, FASTZ_ETRUNC):
         _check(st)
-    rec = np.zeros(max(n.value, 1), dtype=ALIGN_DTYPE)
+    rec = np.empty(max(n.value, 1), dtype=ALIGN_DTYPE)
     cig = ctypes.create_string_buffer(max(nb.value, 1))
     _check(lib().fastz_get_alignments(ctx, rec.ctypes.data, n.value, cig, nb.value, ctypes.byref(n), ctypes.byref(nb)))
     return rec[:n.value], cig.raw[:nb.value]
@@ -243,7 +243,8 @@ class Alignments:
 
     def cigar_of(self, s: int) -> str:
         r = self.rec[s]
-        return self.cigar[r["cigar_off"]: r["cigar_off"] + r["cigar_len"]].decode()
+        c = self.cigar[r["cigar_off"]: r["cigar_off"] + r["cigar_len"]]
+        return (c.tobytes() if isinstance(c, np.ndarray) else c).decode()
 
 
 class Aligner:
@@ -275,6 +276,24 @@ class Aligner:
     def results(self) -> Alignments:
         rec, cig = fastz_get_alignments(self.ctx)
         return Alignments(rec, cig)
+
+    def results_pinned(self) -> Alignments:
+        """Like ``results`` but copies into page-locked host buffers owned by this Aligner and reused by the
+        next call (DMA-speed copies, no page faults); the returned arrays are views valid until then."""
+        import torch
+        n, nb = ctypes.c_int64(), ctypes.c_int64()
+        st = lib().fastz_get_alignments(self.ctx, None, 0, None, 0, ctypes.byref(n), ctypes.byref(nb))
+        if st not in (FASTZ_OK, FASTZ_ETRUNC):
+            _check(st)
+        need_r, need_c = max(n.value, 1) * ALIGN_DTYPE.itemsize, max(nb.value, 1)
+        if getattr(self, "_pin_rec", None) is None or self._pin_rec.numel() < need_r:
+            self._pin_rec = torch.empty(need_r + need_r // 4, dtype=torch.uint8, pin_memory=True)
+        if getattr(self, "_pin_cig", None) is None or self._pin_cig.numel() < need_c:
+            self._pin_cig = torch.empty(need_c + need_c // 4, dtype=torch.uint8, pin_memory=True)
+        _check(lib().fastz_get_alignments(self.ctx, self._pin_rec.data_ptr(), n.value, self._pin_cig.data_ptr(),
+                                          nb.value, ctypes.byref(n), ctypes.byref(nb)))
+        rec = self._pin_rec.numpy()[: n.value * ALIGN_DTYPE.itemsize].view(ALIGN_DTYPE)
+        return Alignments(rec, self._pin_cig.numpy()[: nb.value])
 
     def sides(self):
         return fastz_get_sides(self.ctx, self.n)

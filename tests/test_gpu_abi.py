@@ -88,3 +88,17 @@ def test_repeated_batches_reuse_context():
 def test_int_peak_is_sane():
     ops, mhz = fastz.fastz_int_peak(0, 50.0)
     assert 1e12 < ops < 1e14 and 500 < mhz < 3000
+
+
+def test_results_pinned_equal_results():
+    """Page-locked reusable output buffers (the e2e path of bench.py) give the same records and CIGARs."""
+    w = _w()
+    with fastz.Aligner(w.T, w.Q) as a:
+        r = a.extend(w.seeds)
+        p = a.results_pinned()
+        assert np.array_equal(r.rec, p.rec) and r.cigar == p.cigar.tobytes()
+        assert all(r.cigar_of(s) == p.cigar_of(s) for s in range(0, len(w.seeds), 7))
+        a.extend(w.seeds[:10])           # smaller batch: buffers reused, views shrink
+        p2 = a.results_pinned()
+        assert len(p2.rec) == 10
+        assert all(p2.cigar_of(s) == r.cigar_of(s) for s in range(10))

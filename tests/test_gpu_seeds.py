@@ -55,7 +55,7 @@ def test_edges():
     assert_same(*both("A" * 5000, "C" * 5000))
     rng = np.random.default_rng(5)
     sub = rng.integers(-150, 120, (4, 4))
-    w = genome.small_pair(4, length=8000, n_seeds=8)
+    w = genome.small_pair(4, length=20000, n_seeds=8)
     assert_same(*both(w.T, w.Q, "1101011", True, 300, 200, sub))
 
 
@@ -74,3 +74,30 @@ def test_pipeline_seeds_to_alignments():
     assert len(an) > 5
     bad, g, o, stats = compare(w.T, w.Q, an, census=False)
     assert not bad, bad
+
+
+def revcomp(s: str) -> str:
+    return s.translate(str.maketrans("ACGTacgt", "TGCAtgca"))[::-1]
+
+
+def test_minus_strand():
+    """FASTZ_OPT_QUERY_REVCOMP (32): the context aligns against the reverse complement of the query; HSPs and
+    gapped alignments equal the oracle's on the explicitly reverse-complemented string."""
+    w = genome.small_pair(7, length=30000, n_seeds=8)
+    T = w.T.decode() if isinstance(w.T, bytes) else w.T
+    Q = w.Q.decode() if isinstance(w.Q, bytes) else w.Q
+    Qm = revcomp(T[5000:9000]) + Q[4000:20000] + revcomp(T[15000:17000])  # minus-strand homology
+    rc = revcomp(Qm)
+    with fastz.Aligner(T, Qm, fastz.fastz_default_params(options=32)) as al:
+        g, an, gh = al.find_hsps()
+        ga = al.extend(an)
+    o, oh = seeds.find_hsps(T, rc, core.HOXD70)
+    assert_same(g, an, gh, o, oh)
+    assert len(o) >= 2
+    orr = core.extend(T, rc, an, core.Params())
+    for f in ("score", "t_start", "t_end", "q_start", "q_end"):
+        assert np.array_equal(ga.rec[f].astype(np.int64), orr.rec[f]), f
+    assert all(ga.cigar_of(s) == orr.cigar_of(s) for s in range(len(an)))
+    # invalid character reported at its index in the caller's string
+    with pytest.raises(fastz.FastzError, match="index"):
+        fastz.Aligner(T, Qm[:100] + "N" + Qm[101:], fastz.fastz_default_params(options=32))
