@@ -42,7 +42,7 @@ def full_matrix(A, B, p):
             if i == 0 and j == 0:
                 s, d, ii, c, lv = 0, NEG, NEG, 0, True
             else:
-                h = S[i - 1][j - 1] + p.sub[A[i - 1]][B[j - 1]] if (i >= 1 and j >= 1) else NEG
+                h = S[i - 1][j - 1] + p.s(A[i - 1], B[j - 1]) if (i >= 1 and j >= 1) else NEG
                 d, dbit = NEG, 0
                 if i >= 1:
                     ext, opn = D[i - 1][j] - E, S[i - 1][j] - O - E
@@ -98,7 +98,7 @@ def path_score(A, B, ops, p):
     prev = None
     for op in ops:
         if op == "M":
-            total += p.sub[A[i]][B[j]]
+            total += p.s(A[i], B[j])
             i += 1
             j += 1
         elif op == "D":
@@ -123,7 +123,7 @@ def best_path_score(A, B, p):
         if score > best:
             best = score
         if i < M and j < N:
-            rec(i + 1, j + 1, "M", score + p.sub[A[i]][B[j]])
+            rec(i + 1, j + 1, "M", score + p.s(A[i], B[j]))
         if i < M:
             rec(i + 1, j, "D", score - p.gap_extend - (p.gap_open if prev != "D" else 0))
         if j < N:

@@ -34,15 +34,21 @@ class Params:
     ydrop: int = 9400
     gapped_threshold: int = 3000
     eager_max: int = 16
+    n_score: int = -100   # reading R13: any pair with an N scores n_score (the paper is silent)
+
+    def s(self, a: int, b: int) -> int:
+        """Score of target code a against query code b (A0 C1 G2 T3, N4; reading R13)."""
+        return self.n_score if a == 4 or b == 4 else self.sub[a][b]
 
     def transposed(self) -> "Params":
         return Params(tuple(tuple(self.sub[b][a] for b in range(4)) for a in range(4)),
-                      self.gap_open, self.gap_extend, self.ydrop, self.gapped_threshold, self.eager_max)
+                      self.gap_open, self.gap_extend, self.ydrop, self.gapped_threshold, self.eager_max, self.n_score)
 
 
 class _CParams(ctypes.Structure):
     _fields_ = [("sub", ctypes.c_int32 * 16), ("gap_open", ctypes.c_int32), ("gap_extend", ctypes.c_int32),
-                ("ydrop", ctypes.c_int32), ("gapped_threshold", ctypes.c_int32), ("eager_max", ctypes.c_int32)]
+                ("ydrop", ctypes.c_int32), ("gapped_threshold", ctypes.c_int32), ("eager_max", ctypes.c_int32),
+                ("n_score", ctypes.c_int32)]
 
 
 class _CSide(ctypes.Structure):
@@ -96,10 +102,11 @@ def _cparams(p: Params) -> _CParams:
             c.sub[4 * a + b] = int(p.sub[a][b])
     c.gap_open, c.gap_extend, c.ydrop = int(p.gap_open), int(p.gap_extend), int(p.ydrop)
     c.gapped_threshold, c.eager_max = int(p.gapped_threshold), int(p.eager_max)
+    c.n_score = int(p.n_score)
     return c
 
 
-_CODE = {"A": 0, "C": 1, "G": 2, "T": 3, "a": 0, "c": 1, "g": 2, "t": 3}
+_CODE = {"A": 0, "C": 1, "G": 2, "T": 3, "N": 4, "a": 0, "c": 1, "g": 2, "t": 3, "n": 4}
 
 
 def encode(seq: str) -> np.ndarray:

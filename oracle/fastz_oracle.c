@@ -43,7 +43,13 @@ typedef struct {
     int32_t ydrop;            /* Y >= 0 */
     int32_t gapped_threshold; /* K: flag bit only */
     int32_t eager_max;        /* eager window: classification only */
+    int32_t n_score;          /* reading R13: any pair with an N (code 4) scores n_score */
 } fzo_params;
+
+/* substitution score of target code a against query code b (A0 C1 G2 T3, N4; reading R13) */
+static int64_t subst(const fzo_params *p, int a, int b) {
+    return (a == 4 || b == 4) ? p->n_score : p->sub[4 * a + b];
+}
 
 typedef struct {
     int64_t score, i, j;   /* peak */
@@ -189,7 +195,7 @@ static int one_sided(const uint8_t *A, int64_t M, const uint8_t *B, int64_t N, c
             if (i == 0 && j == 0) {
                 S = 0; D = NEG; I = NEG; code = 0; live = 1;
             } else {
-                int64_t H = (i >= 1 && j >= 1) ? Sd + p->sub[4 * A[i - 1] + B[j - 1]] : NEG;
+                int64_t H = (i >= 1 && j >= 1) ? Sd + subst(p, A[i - 1], B[j - 1]) : NEG;
                 int dbit = 0, ibit = 0;
                 D = NEG;
                 if (i >= 1) {
@@ -263,6 +269,7 @@ static int code_of(char c) {
         case 'C': case 'c': return 1;
         case 'G': case 'g': return 2;
         case 'T': case 't': return 3;
+        case 'N': case 'n': return 4;  /* reading R13 */
         default: return -1;
     }
 }

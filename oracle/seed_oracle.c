@@ -18,6 +18,8 @@
  *   S5 identical HSPs (same t_start, q_start, length) are reported once.
  *   S6 anchor (the gapped extension's cut point): the HSP midpoint t_start + length/2, q_start + length/2.
  *      Output sorted by (anchor t, anchor q, t_start, length).
+ *   S7 N (code 4): a word with an N at a care position matches nothing; in the walks any pair with an N scores
+ *      n_score (reading R13).
  * Written for clarity: a sorted (word, position) index of T, a binary search per query word and variant, one
  * loop per extension.  No blocking, no fusion.
  */
@@ -41,6 +43,7 @@ static int code_of(char c) {
         case 'C': case 'c': return 1;
         case 'G': case 'g': return 2;
         case 'T': case 't': return 3;
+        case 'N': case 'n': return 4;
         default: return -1;
     }
 }
@@ -71,17 +74,27 @@ static int cmp_hsp_anchor(const void* a, const void* b) {
     return x->length < y->length ? -1 : (x->length > y->length);
 }
 
-/* S1: word at position p (care offsets off[0..w-1]), 2 bits per care position, first care position highest */
-static uint32_t word_at(const int8_t* s, int64_t p, const int* off, int w) {
+/* S1: word at position p (care offsets off[0..w-1]), 2 bits per care position, first care position highest.
+ * S7: *valid = 0 if a care position holds an N. */
+static uint32_t word_at(const int8_t* s, int64_t p, const int* off, int w, int* valid) {
     uint32_t k = 0;
-    for (int c = 0; c < w; ++c) k = (k << 2) | (uint32_t)s[p + off[c]];
+    *valid = 1;
+    for (int c = 0; c < w; ++c) {
+        if (s[p + off[c]] == 4) *valid = 0;
+        k = (k << 2) | (uint32_t)(s[p + off[c]] & 3);
+    }
     return k;
+}
+
+/* reading R13: any pair with an N scores n_score */
+static int64_t subst(const int32_t* sub16, int32_t n_score, int a, int b) {
+    return (a == 4 || b == 4) ? n_score : sub16[4 * a + b];
 }
 
 /* Returns 0, -1 (bad argument), -2 (bad base), -4 (out of memory), -6 (out buffer too small: *n_out = needed). */
 int fzs_find(const char* T, int64_t tlen, const char* Q, int64_t qlen, const char* pattern, int transitions,
-             const int32_t* sub16, int32_t xdrop, int32_t hspthresh, fzs_hsp* out, int64_t cap, int64_t* n_out,
-             int64_t* n_hits) {
+             const int32_t* sub16, int32_t n_score, int32_t xdrop, int32_t hspthresh, fzs_hsp* out, int64_t cap,
+             int64_t* n_out, int64_t* n_hits) {
     const int L = (int)strlen(pattern);
     int off[32], w = 0;
     if (L < 1 || L > 64 || xdrop < 0) return -1;
@@ -103,34 +116,41 @@ int fzs_find(const char* T, int64_t tlen, const char* Q, int64_t qlen, const cha
     /* index of T: (word, position) sorted */
     const int64_t nt = tlen >= L ? tlen - L + 1 : 0;
     kp* idx = (kp*)malloc(sizeof(kp) * (size_t)(nt + 1));
+    int64_t ni = 0;
     for (int64_t p = 0; p < nt; ++p) {
-        idx[p].key = word_at(t, p, off, w);
-        idx[p].pos = p;
+        int valid;
+        const uint32_t k = word_at(t, p, off, w, &valid);
+        if (!valid) continue; /* S7 */
+        idx[ni].key = k;
+        idx[ni].pos = p;
+        ++ni;
     }
-    qsort(idx, (size_t)nt, sizeof(kp), cmp_kp);
+    qsort(idx, (size_t)ni, sizeof(kp), cmp_kp);
 
     int64_t hcap = 1024, nh = 0, hits = 0;
     fzs_hsp* hs = (fzs_hsp*)malloc(sizeof(fzs_hsp) * (size_t)hcap);
     const int64_t nq = qlen >= L ? qlen - L + 1 : 0;
     for (int64_t qp = 0; qp < nq; ++qp) {
-        const uint32_t k0 = word_at(q, qp, off, w);
+        int valid;
+        const uint32_t k0 = word_at(q, qp, off, w, &valid);
+        if (!valid) continue; /* S7 */
         const int nvar = transitions ? 1 + w : 1;
         for (int v = 0; v < nvar; ++v) {
             /* S2: variant 0 = exact word; variant 1 + c = transition at care position c (A<->G, C<->T: xor 2) */
             const uint32_t k = v == 0 ? k0 : k0 ^ (2u << (2 * (w - v)));
             /* binary search for the first index entry with this key */
-            int64_t lo = 0, hi = nt;
+            int64_t lo = 0, hi = ni;
             while (lo < hi) {
                 const int64_t mid = (lo + hi) / 2;
                 if (idx[mid].key < k) lo = mid + 1; else hi = mid;
             }
-            for (int64_t e = lo; e < nt && idx[e].key == k; ++e) {
+            for (int64_t e = lo; e < ni && idx[e].key == k; ++e) {
                 const int64_t tp = idx[e].pos;
                 ++hits;
                 /* S3: right extension */
                 int64_t s = 0, best_r = 0, r = 0;
                 for (int64_t d = 0; tp + d < tlen && qp + d < qlen; ++d) {
-                    s += sub16[4 * t[tp + d] + q[qp + d]];
+                    s += subst(sub16, n_score, t[tp + d], q[qp + d]);
                     if (s > best_r) {
                         best_r = s;
                         r = d + 1;
@@ -141,7 +161,7 @@ int fzs_find(const char* T, int64_t tlen, const char* Q, int64_t qlen, const cha
                 int64_t best_l = 0, l = 0;
                 s = 0;
                 for (int64_t d = 1; tp - d >= 0 && qp - d >= 0; ++d) {
-                    s += sub16[4 * t[tp - d] + q[qp - d]];
+                    s += subst(sub16, n_score, t[tp - d], q[qp - d]);
                     if (s > best_l) {
                         best_l = s;
                         l = d;

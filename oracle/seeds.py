@@ -45,7 +45,7 @@ def lib():
         _lib = ctypes.CDLL(build())
         _lib.fzs_find.restype = ctypes.c_int
         _lib.fzs_find.argtypes = [ctypes.c_char_p, ctypes.c_int64, ctypes.c_char_p, ctypes.c_int64, ctypes.c_char_p,
-                                  ctypes.c_int, ctypes.POINTER(ctypes.c_int32), ctypes.c_int32, ctypes.c_int32,
+                                  ctypes.c_int, ctypes.POINTER(ctypes.c_int32), ctypes.c_int32, ctypes.c_int32, ctypes.c_int32,
                                   ctypes.c_void_p, ctypes.c_int64, ctypes.POINTER(ctypes.c_int64),
                                   ctypes.POINTER(ctypes.c_int64)]
     return _lib
@@ -56,7 +56,7 @@ def _sub16(sub) -> ctypes.Array:
 
 
 def find_hsps(T, Q, sub, pattern: str = PATTERN_12OF19, transitions: bool = True, xdrop: int = XDROP,
-              hspthresh: int = HSPTHRESH):
+              hspthresh: int = HSPTHRESH, n_score: int = -100):
     """HSPs (structured array, HSP_DTYPE) in anchor order, and the raw hit count."""
     T = T.encode() if isinstance(T, str) else bytes(T)
     Q = Q.encode() if isinstance(Q, str) else bytes(Q)
@@ -66,7 +66,7 @@ def find_hsps(T, Q, sub, pattern: str = PATTERN_12OF19, transitions: bool = True
         out = np.zeros(cap, dtype=HSP_DTYPE)
         n = ctypes.c_int64(0)
         hits = ctypes.c_int64(0)
-        rc = L.fzs_find(T, len(T), Q, len(Q), pattern.encode(), int(transitions), _sub16(sub), xdrop, hspthresh,
+        rc = L.fzs_find(T, len(T), Q, len(Q), pattern.encode(), int(transitions), _sub16(sub), n_score, xdrop, hspthresh,
                         out.ctypes.data, cap, ctypes.byref(n), ctypes.byref(hits))
         if rc == -6:
             cap = int(n.value)
@@ -76,7 +76,7 @@ def find_hsps(T, Q, sub, pattern: str = PATTERN_12OF19, transitions: bool = True
         return out[: n.value].copy(), int(hits.value)
 
 
-_CODE = {"A": 0, "C": 1, "G": 2, "T": 3}
+_CODE = {"A": 0, "C": 1, "G": 2, "T": 3, "N": 4}
 _TRANSITION = {("A", "G"), ("G", "A"), ("C", "T"), ("T", "C")}
 
 
@@ -88,19 +88,21 @@ def brute_hits(T: str, Q: str, pattern: str = PATTERN_12OF19, transitions: bool 
     hits = []
     for t in range(len(T) - L + 1):
         for q in range(len(Q) - L + 1):
+            if any(T[t + c] == "N" or Q[q + c] == "N" for c in care):  # S7
+                continue
             diff = [(T[t + c], Q[q + c]) for c in care if T[t + c] != Q[q + c]]
             if not diff or (transitions and len(diff) == 1 and diff[0] in _TRANSITION):
                 hits.append((t, q))
     return hits
 
 
-def ungapped(T: str, Q: str, t: int, q: int, sub, xdrop: int = XDROP):
-    """S3 for one hit: (t_start, q_start, length, score)."""
+def ungapped(T: str, Q: str, t: int, q: int, sub, xdrop: int = XDROP, n_score: int = -100):
+    """S3 for one hit: (t_start, q_start, length, score); an N scores n_score (S7)."""
     T, Q = T.upper(), Q.upper()
     def walk(pairs):
         s = best = ext = 0
         for d, (a, b) in enumerate(pairs, 1):
-            s += sub[_CODE[a]][_CODE[b]]
+            s += n_score if "N" in (a, b) else sub[_CODE[a]][_CODE[b]]
             if s > best:
                 best, ext = s, d
             if s < best - xdrop:
@@ -112,9 +114,9 @@ def ungapped(T: str, Q: str, t: int, q: int, sub, xdrop: int = XDROP):
 
 
 def brute_hsps(T: str, Q: str, sub, pattern: str = PATTERN_12OF19, transitions: bool = True, xdrop: int = XDROP,
-               hspthresh: int = HSPTHRESH):
+               hspthresh: int = HSPTHRESH, n_score: int = -100):
     """S2-S6 by brute force: every hit extended, filtered, deduplicated, sorted by anchor."""
-    hs = {ungapped(T, Q, t, q, sub, xdrop) for t, q in brute_hits(T, Q, pattern, transitions)}
+    hs = {ungapped(T, Q, t, q, sub, xdrop, n_score) for t, q in brute_hits(T, Q, pattern, transitions)}
     hs = [h for h in hs if h[3] >= hspthresh]
     hs.sort(key=lambda h: (h[0] + h[2] // 2, h[1] + h[2] // 2, h[0], h[2]))
     return hs

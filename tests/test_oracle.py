@@ -269,6 +269,40 @@ def test_flags_and_eager():
 
 def test_bad_inputs():
     with pytest.raises(RuntimeError):
-        core.extend("ACGN", "ACGT", [(1, 1)])
+        core.extend("ACGX", "ACGT", [(1, 1)])
     with pytest.raises(RuntimeError):
         core.extend("ACGT", "ACGT", [(5, 1)])
+
+
+# ---------------------------------------------------------------- N bases (reading R13, NEXT-4)
+
+
+def test_n_closed_form():
+    """An N scores n_score against anything: ACNGT vs ACNGT = 91 + 100 + n + 100 + 91, all matches."""
+    for n in (-100, 0):
+        p = dataclasses.replace(P0, n_score=n)
+        s = core.one_sided("ACNGT", "ACNGT", p)
+        assert (s.score, s.i, s.j, s.ops) == (382 + n, 5, 5, "M" * 5)
+    # n = -1000: crossing the N (191 - 1000 + 191 < 191) loses to stopping before it; skipping it costs two
+    # gap opens (-860), so the peak is (191, 2, 2)
+    s = core.one_sided("ACNGT", "ACNGT", dataclasses.replace(P0, n_score=-1000))
+    assert (s.score, s.i, s.j, s.ops) == (191, 2, 2, "MM")
+    # a deep N run breaks the extension exactly like mismatches of the same score would
+    p = dataclasses.replace(P0, n_score=-114)
+    a = "A" * 20 + "N" * 10 + "A" * 20
+    b = "A" * 20 + "C" * 10 + "A" * 20
+    assert core.one_sided(a, "A" * 50, p).score == core.one_sided(b, "A" * 50, P0).score  # sub(C, A) = -114
+
+
+def test_n_full_matrix_and_paths():
+    """Random sequences with N on both sides: banded oracle == full matrix; exhaustive paths == peak."""
+    rng = random.Random(4242)
+    nseq = lambda k: "".join(rng.choice("ACGTN") for _ in range(k))
+    for _ in range(60):
+        p = dataclasses.replace(rand_params(rng), n_score=rng.choice([-100, -7, 0, 25]))
+        _cmp_full(nseq(rng.randint(0, 40)), nseq(rng.randint(0, 40)), p)
+    for trial in range(80):
+        p = dataclasses.replace(rand_params(rng), ydrop=10 ** 8, n_score=rng.choice([-100, 0, 40]))
+        a, b = nseq(rng.randint(0, 6)), nseq(rng.randint(0, 6))
+        s = core.one_sided(a, b, p)
+        assert s.score == brute.best_path_score(core.encode(a), core.encode(b), p), (trial, a, b)

@@ -112,6 +112,29 @@ def test_anchor_order_and_dedup():
 
 def test_bad_input():
     with pytest.raises(ValueError):
-        seeds.find_hsps("ACGN" * 10, "ACGT" * 10, HOXD70)
+        seeds.find_hsps("ACGX" * 10, "ACGT" * 10, HOXD70)
     with pytest.raises(ValueError):
         seeds.find_hsps("ACGT" * 10, "ACGT" * 10, HOXD70, pattern="0110")
+
+
+def test_n_bases():
+    """S7: words with an N at a care position match nothing; walks score N as n_score.  Brute force agrees."""
+    rng = np.random.default_rng(77)
+    for trial in range(4):
+        core_ = rand_seq(160, rng)
+        T = list(rand_seq(30, rng) + core_ + rand_seq(30, rng))
+        Q = list(rand_seq(20, rng) + mutate(core_, rng) + rand_seq(40, rng))
+        for s_ in (T, Q):
+            for p in rng.choice(len(s_), 6, replace=False):
+                s_[p] = "N"
+        T, Q = "".join(T), "".join(Q)
+        for pattern, nsc in ((seeds.PATTERN_12OF19, -100), ("1101011", 0), ("111", -300)):
+            got, hits = seeds.find_hsps(T, Q, HOXD70, pattern, True, 910, 300, nsc)
+            assert as_tuples(got) == seeds.brute_hsps(T, Q, HOXD70, pattern, True, 910, 300, nsc)
+            assert hits == len(seeds.brute_hits(T, Q, pattern, True))
+    # an N at a don't-care position does not block a hit; at a care position it does
+    base = rand_seq(19, rng)
+    dont = seeds.PATTERN_12OF19.index("0")
+    care = seeds.PATTERN_12OF19.index("1")
+    assert (0, 0) in seeds.brute_hits(base, base[:dont] + "N" + base[dont + 1:])
+    assert (0, 0) not in seeds.brute_hits(base, base[:care] + "N" + base[care + 1:])
