@@ -465,13 +465,21 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     }
     AL(codes, std::max<long long>(pool_words, 1) * 4);
     Outputs o = make_out(c);
+    // executor timing starts here: the host sync + pool sizing above count to the binning stage
+    CK(cudaEventRecord(c->ev[7], st));
+    int64_t tb_launches = 0;  // per wave: warp-per-side (list positions < nblock) and thread-per-side launches
     for (size_t w = 0; w < waves.size(); ++w) {
+        {
+            const long long lo = waves[w].first, hi = waves[w].second;
+            const long long mid = std::min(std::max(nblock, lo), hi);
+            tb_launches += (mid > lo ? 1 : 0) + (hi > mid ? 1 : 0);
+        }
         if (w) CK(cudaMemsetAsync(P_<int>(c->counters) + 1, 0, 4, st));
         if (w) CK(cudaMemsetAsync(P_<int>(c->counters) + 23, 0, 4, st));
         CK(launch_execute(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, (int)waves[w].first,
                           (int)waves[w].second, (int)nblock, wbase[w], o, st));
         if (w == 0) CK(cudaEventRecord(c->ev[4], st));
-        CK(launch_traceback(c->R, sa, pl, (int)waves[w].first, (int)waves[w].second, wbase[w], o, st));
+        CK(launch_traceback(c->R, sa, pl, (int)waves[w].first, (int)waves[w].second, (int)nblock, wbase[w], o, st));
     }
     if (waves.empty()) CK(cudaEventRecord(c->ev[4], st));
     CK(cudaEventRecord(c->ev[5], st));
@@ -500,8 +508,9 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     S.n_waves = c->nwaves;
     S.n_escalated = h.counters[21];
     // own kernels: validate, inspect, inspect_block (if escalation on), bin_count, bin_offsets, bin_scatter,
-    // list_words, list_offsets, execute + traceback per wave, combine_len, combine_total, combine_write
-    S.n_launches = (n > 0 ? 1 + 1 + (esc > 0 ? 1 : 0) + 5 + 2 * (int64_t)c->nwaves + 3 : 1);
+    // list_words, list_offsets, execute per wave, traceback (warp and/or thread variant) per wave, combine_len,
+    // combine_total, combine_write
+    S.n_launches = (n > 0 ? 1 + 1 + (esc > 0 ? 1 : 0) + 5 + (int64_t)c->nwaves + tb_launches + 3 : 1);
     c->have = true;
     return 0;
 }
@@ -579,8 +588,8 @@ int fastz_get_stats(fastz_ctx* c, fastz_stats* s) {
     };
     S.ms_upload = el(0, 1);
     S.ms_inspect = el(1, 2);
-    S.ms_bin = el(2, 3);
-    S.ms_execute = el(3, 4);
+    S.ms_bin = el(2, 7);      // binning kernels + host sync 1 + traceback-pool sizing
+    S.ms_execute = el(7, 4);
     S.ms_traceback = el(4, 5);
     S.ms_combine = el(5, 6);
     S.ms_total = el(0, 6);

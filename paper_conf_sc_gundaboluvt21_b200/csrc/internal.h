@@ -76,8 +76,8 @@ cudaError_t launch_execute(int R, int grid, const DevParams& P, const Batch& b, 
                            const SideArrays& sa, const ExecPlan& pl, int lo, int hi, int nblock, long long base,
                            const Outputs& o,
                            cudaStream_t st);
-cudaError_t launch_traceback(int R, const SideArrays& sa, const ExecPlan& pl, int lo, int hi, long long base,
-                             const Outputs& o, cudaStream_t st);
+cudaError_t launch_traceback(int R, const SideArrays& sa, const ExecPlan& pl, int lo, int hi, int nblock,
+                             long long base, const Outputs& o, cudaStream_t st);
 cudaError_t launch_combine_len(const DevParams& P, const Batch& b, const SideArrays& sa, const ExecPlan& pl,
                                const Outputs& o, void* scan_tmp, size_t scan_tmp_bytes, long long* total,
                                cudaStream_t st);

@@ -395,6 +395,75 @@ __global__ void k_traceback(SideArrays sa, ExecPlan pl, int lo, int hi, long lon
     out.nruns[side] = nr;
 }
 
+// Warp per side (long sides, list positions < nblock = bins >= 3): the walk is the same chain of dependent
+// steps, but the code words come from a shared-memory window that the warp refills with coalesced loads (64
+// word rows = 8 KB per warp: the next 64 * SPW steps to the left of the current one in the strip), so a
+// step costs a shared-memory read instead of an HBM round trip.  All 32 lanes walk in lockstep (uniform control
+// flow); lane 0 writes the runs.
+constexpr int TBW_ROWS = 64;  // word rows (32 words each) per window
+template <int R>
+__global__ void __launch_bounds__(128) k_traceback_warp(SideArrays sa, ExecPlan pl, int lo, int hi, long long base,
+                                                        Outputs out) {
+    constexpr int H = 32 * R, SPW = 8 / R;
+    __shared__ uint32_t win[4][TBW_ROWS * 32];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int idx = lo + blockIdx.x * 4 + warp;
+    if (idx >= hi) return;
+    uint32_t* wbuf = win[warp];
+    const int side = pl.list[idx];
+    const uint32_t* __restrict__ codes = out.codes + (pl.woff[side] - base);
+    const int2* __restrict__ stab = out.stab + pl.soff[side];
+    uint32_t* __restrict__ runs = out.runs + pl.roff[side];
+    int i = sa.ti[side], j = sa.qj[side], state = 0, nr = 0;
+    uint32_t cur = 0xffffffffu, len = 0;
+    auto emit = [&](uint32_t op) {
+        if (op == cur) {
+            ++len;
+        } else {
+            if (len && lane == 0) runs[nr] = (len << 2) | cur;
+            nr += len ? 1 : 0;
+            cur = op;
+            len = 1;
+        }
+    };
+    int scur = -1, rlo = 0, rhi = 0;  // window = word rows [rlo, rhi) of strip scur
+    int2 st = make_int2(0, 0);
+    while (i > 0 || j > 0) {
+        const int s = i / H, lr = i - s * H, ln = lr / R, k = lr - ln * R;
+        if (s != scur) {
+            st = stab[s];
+            scur = s;
+            rhi = 0;
+            rlo = 1;  // empty
+        }
+        const int t = j - st.x + ln;
+        const int wr = t / SPW;
+        if (wr < rlo || wr >= rhi) {  // refill: rows [wr - TBW_ROWS + 1, wr] (the walk moves to smaller t)
+            rhi = wr + 1;
+            rlo = rhi - TBW_ROWS > 0 ? rhi - TBW_ROWS : 0;
+            __syncwarp();
+            const uint32_t* src = codes + (long long)st.y + (long long)rlo * 32 + lane;
+#pragma unroll 8
+            for (int r = 0; r < rhi - rlo; ++r) wbuf[r * 32 + lane] = src[(long long)r * 32];
+            __syncwarp();
+        }
+        const uint32_t w = wbuf[(wr - rlo) * 32 + ln];
+        const uint32_t code = (w >> ((((t % SPW) * R) + k) * 4)) & 15u;
+        const int eff = state == 0 ? (int)(code & 3u) : state;  // 0 M, 1 D, 2 I
+        const uint32_t op = eff == 0 ? (uint32_t)OP_M : (eff == 1 ? (uint32_t)OP_D : (uint32_t)OP_I);
+        const bool ext = eff == 1 ? ((code >> 2) & 1u) : ((code >> 3) & 1u);
+        state = eff == 0 ? 0 : (ext ? eff : 0);
+        i -= eff != 2;
+        j -= eff != 1;
+        emit(op);
+    }
+    if (len) {
+        if (lane == 0) runs[nr] = (len << 2) | cur;
+        ++nr;
+    }
+    if (lane == 0) out.nruns[side] = nr;
+}
+
 // ------------------------------------------------------------------------------------------------- binning
 // Bins by max(i*, j*) (512, 2048, 8192, 32768, then 4x): bin 0 = eager.
 __device__ __forceinline__ int bin_of(int m) {
@@ -703,12 +772,21 @@ cudaError_t launch_execute(int R, int grid, const DevParams& P, const Batch& b, 
     return cudaGetLastError();
 }
 
-cudaError_t launch_traceback(int R, const SideArrays& sa, const ExecPlan& pl, int lo, int hi, long long base,
-                             const Outputs& o, cudaStream_t st) {
+cudaError_t launch_traceback(int R, const SideArrays& sa, const ExecPlan& pl, int lo, int hi, int nblock,
+                             long long base, const Outputs& o, cudaStream_t st) {
     if (hi <= lo) return cudaSuccess;
-    const int g = (hi - lo + 127) / 128;
-    if (R == 2) k_traceback<2><<<g, 128, 0, st>>>(sa, pl, lo, hi, base, o);
-    else k_traceback<4><<<g, 128, 0, st>>>(sa, pl, lo, hi, base, o);
+    // list positions < nblock hold the long sides (bins >= 3): warp per side with a shared code window
+    const int mid = nblock < lo ? lo : (nblock > hi ? hi : nblock);
+    if (mid > lo) {
+        const int g = (mid - lo + 3) / 4;
+        if (R == 2) k_traceback_warp<2><<<g, 128, 0, st>>>(sa, pl, lo, mid, base, o);
+        else k_traceback_warp<4><<<g, 128, 0, st>>>(sa, pl, lo, mid, base, o);
+    }
+    if (hi > mid) {
+        const int g = (hi - mid + 127) / 128;
+        if (R == 2) k_traceback<2><<<g, 128, 0, st>>>(sa, pl, mid, hi, base, o);
+        else k_traceback<4><<<g, 128, 0, st>>>(sa, pl, mid, hi, base, o);
+    }
     return cudaGetLastError();
 }
 

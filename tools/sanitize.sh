@@ -1,4 +1,5 @@
 # compute-sanitizer on a small mixed workload (memcheck, racecheck, synccheck, initcheck); block-per-side forced
+# (so the warp-per-side traceback runs too), plus the seeding stage on both strands
 mkdir -p gpurun_out
 python -m paper_conf_sc_gundaboluvt21_b200.build > /dev/null
 cat > /tmp/san_case.py <<'PY'
@@ -10,7 +11,11 @@ w = genome.small_pair(90, length=8000, n_seeds=40)
 with fastz.Aligner(w.T, w.Q) as a:
     r = a.extend(w.seeds)
     a.census()
-print("ok", len(r.rec))
+    hs, an, hits = a.find_hsps(hspthresh=500)
+    a.extend(an)
+with fastz.Aligner(w.T, w.Q, fastz.fastz_default_params(options=32)) as b:
+    hs2, an2, _ = b.find_hsps(pattern="1101011", hspthresh=300)
+print("ok", len(r.rec), len(hs), len(hs2))
 PY
 for tool in memcheck racecheck synccheck initcheck; do
   FASTZ_ESCALATE_STRIPS=2 FASTZ_BLOCK_BIN=1 timeout 900 compute-sanitizer --tool $tool --error-exitcode 9 python /tmp/san_case.py > gpurun_out/san_$tool.log 2>&1; echo "$tool rc=$?"; tail -2 gpurun_out/san_$tool.log
