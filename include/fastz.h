@@ -37,7 +37,7 @@ typedef struct fastz_ctx fastz_ctx; /* opaque */
 typedef enum {
     FASTZ_OK = 0,
     FASTZ_EINVAL = -1, /* bad argument or scoring parameter (ranges below) */
-    FASTZ_EBASE = -2,  /* a sequence character outside ACGTacgt (index in fastz_strerror text) */
+    FASTZ_EBASE = -2,  /* a sequence character outside ACGTNacgtn (index in fastz_strerror text) */
     FASTZ_ERANGE = -3, /* seed outside [0,len]; length >= 2^31; an explored band wider than the scratch */
     FASTZ_ENOMEM = -4, /* device allocation failed */
     FASTZ_ECUDA = -5,  /* CUDA runtime error (text in fastz_strerror) */
@@ -57,6 +57,8 @@ typedef enum {
  *   gapped_threshold  K: only sets FASTZ_FLAG_ABOVE_K; never drops a seed.
  *   eager_max   eager-traceback window, 1..16 (16x16); sides whose peak has max(i*,j*) <= eager_max
  *               are traced back inside the inspector and skip the executor.
+ *   n_score     N (unknown base, either case) in either sequence scores n_score against anything; default -100
+ *               (reading R13; the paper is silent).  Spaced seeds never match across an N (S7).
  *   dev_alloc / dev_free / alloc_user  optional device allocator hooks (e.g. a framework caching
  *               allocator); NULL -> cudaMalloc / cudaFree.
  */
@@ -68,7 +70,8 @@ typedef struct {
     int32_t gapped_threshold;
     int32_t eager_max;
     int32_t options;              /* FASTZ_OPT_* bits, 0 = the paper's full design (see below) */
-    int32_t reserved[2];
+    int32_t n_score;              /* score of any pair with an N (either sequence), |n_score| <= 32767 */
+    int32_t reserved;
     void *(*dev_alloc)(size_t bytes, void *stream, void *user);
     void (*dev_free)(void *ptr, void *stream, void *user);
     void *alloc_user;
@@ -116,9 +119,9 @@ void fastz_default_params(fastz_params *p);
 
 /*
  * Create a context on `device` using `cuda_stream` (a cudaStream_t; NULL -> the library creates its own
- * non-blocking stream).  `target`/`query` are ASCII (ACGTacgt) of tlen/qlen bytes, host or device memory
+ * non-blocking stream).  `target`/`query` are ASCII (ACGTNacgtn) of tlen/qlen bytes, host or device memory
  * (detected with cudaPointerGetAttributes); they are copied, validated and packed to 2 bits per base
- * (forward and reversed copies) on the device.  Errors: EINVAL (NULL pointers, bad params), ERANGE (a length
+ * (forward and reversed copies) plus a 1-bit N mask on the device.  Errors: EINVAL (NULL pointers, bad params), ERANGE (a length
  * < 0 or >= 2^31), EBASE (invalid character), ENOMEM, ECUDA.  On error *out is NULL.
  */
 int fastz_create(const fastz_params *p, const char *target, int64_t tlen, const char *query, int64_t qlen,

@@ -23,6 +23,7 @@
  *   R6 extension ends at the first row without a live cell ("if all the scores of a row fall below").
  *   R7 explored cells (the GCUPS numerator) = origin + cells with a live diagonal/up/left predecessor.
  *   R8 peak scores >= 2^29 are flagged (score range of the int32 ABI), not an error of the method.
+ *   R13 N (code 4, either sequence) scores n_score against anything; other non-ACGT characters are errors.
  *
  * Plain row-major scan; int64 arithmetic; one byte per traceback code (bits 1:0 = S source 0 H/1 D/2 I,
  * bit 2 = D extends, bit 3 = I extends -- P:178's 2+1+1 bits).  V(i-1, j) is obtained from a per-column

@@ -52,6 +52,8 @@ struct fastz_ctx {
     DevParams dp{};
     int tlen = 0, qlen = 0;
     DBuf Tf, Tr, Qf, Qr, stage;
+    DBuf TfN, TrN, QfN, QrN;  // N masks (1 bit per base, 16 per u16 word)
+    bool t_has_n = false, q_has_n = false;
     DBuf seeds, score, ti, qj, flags, eops, bound, maxsw, esc, nstrip;
     DBuf woff, soff, roff, bin, list, counters, totals, tmpa, tmpb, tmpc, scan_tmp, wl, wlo;
     DBuf codes, stab, runs, nruns, ciglen, cigar, recs, cells, ring, small;
@@ -127,6 +129,7 @@ int check_params(const fastz_params* p) {
     if (!p) return fail(FASTZ_EINVAL, "params is NULL");
     for (int k = 0; k < 16; ++k)
         if (p->sub[k] < -32767 || p->sub[k] > 32767) return fail(FASTZ_EINVAL, "|sub| must be <= 32767");
+    if (p->n_score < -32767 || p->n_score > 32767) return fail(FASTZ_EINVAL, "|n_score| must be <= 32767");
     if (p->gap_open < 0 || p->gap_open > (1 << 24)) return fail(FASTZ_EINVAL, "gap_open must be in [0, 2^24]");
     if (p->gap_extend < 1 || p->gap_extend > (1 << 24)) return fail(FASTZ_EINVAL, "gap_extend must be in [1, 2^24]");
     if (p->ydrop < 0 || p->ydrop > (1 << 28)) return fail(FASTZ_EINVAL, "ydrop must be in [0, 2^28]");
@@ -134,13 +137,19 @@ int check_params(const fastz_params* p) {
     return 0;
 }
 
-int upload_seq(fastz_ctx* c, const char* src, int64_t len, DBuf& fwd, DBuf& rev, int64_t base_index, int revcomp) {
+int upload_seq(fastz_ctx* c, const char* src, int64_t len, DBuf& fwd, DBuf& rev, DBuf& fwdn, DBuf& revn,
+               bool& has_n, int64_t base_index, int revcomp) {
     const size_t words = (size_t)((len + 15) / 16) + 4;
     int r;
     if ((r = dalloc(c, fwd, words * 4))) return r;
     if ((r = dalloc(c, rev, words * 4))) return r;
+    if ((r = dalloc(c, fwdn, words * 2))) return r;
+    if ((r = dalloc(c, revn, words * 2))) return r;
     CK(cudaMemsetAsync(fwd.p, 0, words * 4, c->stream));
     CK(cudaMemsetAsync(rev.p, 0, words * 4, c->stream));
+    CK(cudaMemsetAsync(fwdn.p, 0, words * 2, c->stream));
+    CK(cudaMemsetAsync(revn.p, 0, words * 2, c->stream));
+    has_n = false;
     if (len == 0) return 0;
     const char* dsrc = src;
     if (!is_device_ptr(src)) {
@@ -149,12 +158,15 @@ int upload_seq(fastz_ctx* c, const char* src, int64_t len, DBuf& fwd, DBuf& rev,
         dsrc = P_<char>(c->stage);
     }
     if ((r = dalloc(c, c->small, 64))) return r;
-    long long init = LLONG_MAX;
-    CK(cudaMemcpyAsync(c->small.p, &init, sizeof(init), cudaMemcpyHostToDevice, c->stream));
-    CK(launch_pack(dsrc, len, P_<uint32_t>(fwd), P_<uint32_t>(rev), P_<long long>(c->small), revcomp, c->stream));
-    long long bad = 0;
-    CK(cudaMemcpyAsync(&bad, c->small.p, sizeof(bad), cudaMemcpyDeviceToHost, c->stream));
+    long long init[2] = {LLONG_MAX, 0};  // first invalid character, has-N flag
+    CK(cudaMemcpyAsync(c->small.p, init, sizeof(init), cudaMemcpyHostToDevice, c->stream));
+    CK(launch_pack(dsrc, len, P_<uint32_t>(fwd), P_<uint32_t>(rev), P_<uint16_t>(fwdn), P_<uint16_t>(revn),
+                   P_<long long>(c->small), revcomp, c->stream));
+    long long res[2] = {0, 0};
+    CK(cudaMemcpyAsync(res, c->small.p, sizeof(res), cudaMemcpyDeviceToHost, c->stream));
     CK(cudaStreamSynchronize(c->stream));
+    const long long bad = res[0];
+    has_n = res[1] != 0;
     if (bad != LLONG_MAX)
         return fail(FASTZ_EBASE, "invalid base character at index " + std::to_string(base_index + bad) +
                                      (base_index ? " (query offset " + std::to_string(bad) + ")" : " (target)"));
@@ -173,6 +185,10 @@ Batch make_batch(fastz_ctx* c) {
     b.Tr = P_<uint32_t>(c->Tr);
     b.Qf = P_<uint32_t>(c->Qf);
     b.Qr = P_<uint32_t>(c->Qr);
+    b.TfN = c->t_has_n ? P_<uint16_t>(c->TfN) : nullptr;
+    b.TrN = c->t_has_n ? P_<uint16_t>(c->TrN) : nullptr;
+    b.QfN = c->q_has_n ? P_<uint16_t>(c->QfN) : nullptr;
+    b.QrN = c->q_has_n ? P_<uint16_t>(c->QrN) : nullptr;
     b.tlen = c->tlen;
     b.qlen = c->qlen;
     b.seeds = P_<long long>(c->seeds);
@@ -242,6 +258,7 @@ void fastz_default_params(fastz_params* p) {
     p->ydrop = 9400;
     p->gapped_threshold = 3000;
     p->eager_max = 16;
+    p->n_score = -100;  // reading R13
 }
 
 void fastz_default_seed_params(fastz_seed_params* sp) {
@@ -274,7 +291,7 @@ void fastz_destroy(fastz_ctx* c) {
     if (!c) return;
     cudaSetDevice(c->device);
     if (c->stream) cudaStreamSynchronize(c->stream);
-    DBuf* bufs[] = {&c->Tf, &c->Tr, &c->Qf, &c->Qr, &c->stage, &c->seeds, &c->score, &c->ti, &c->qj,
+    DBuf* bufs[] = {&c->Tf, &c->Tr, &c->Qf, &c->Qr, &c->TfN, &c->TrN, &c->QfN, &c->QrN, &c->stage, &c->seeds, &c->score, &c->ti, &c->qj,
                     &c->flags, &c->eops, &c->bound, &c->maxsw, &c->esc, &c->nstrip, &c->woff, &c->soff, &c->roff, &c->bin, &c->list,
                     &c->counters, &c->totals, &c->tmpa, &c->tmpb, &c->tmpc, &c->scan_tmp, &c->wl, &c->wlo, &c->codes,
                     &c->stab, &c->runs, &c->nruns, &c->ciglen, &c->cigar, &c->recs, &c->cells, &c->ring,
@@ -311,13 +328,18 @@ int fastz_create(const fastz_params* p, const char* target, int64_t tlen, const 
         }
         c->own_stream = true;
     }
-    // substitution table with O+E folded in (H = X_diag + v is one FMA-pipe IMAD); column code 4 = the origin
-    // column (sub = 0)
+    // substitution table with O+E folded in (H = X_diag + v is one FMA-pipe IMAD): sv[5 * code + a], column
+    // code 0..3 = query base, 4 = the origin column (sub = 0), 5 = N; target base a = 0..3, 4 = N (R13)
     {
         const int oe = p->gap_open + p->gap_extend;
-        for (int b = 0; b < 4; ++b)
-            for (int a = 0; a < 4; ++a) c->dp.sv[4 * b + a] = p->sub[4 * a + b] + oe;
-        for (int a = 0; a < 4; ++a) c->dp.sv[16 + a] = oe;
+        for (int code = 0; code < 6; ++code)
+            for (int a = 0; a < 5; ++a) {
+                int v;
+                if (code == 4) v = 0;
+                else if (code == 5 || a == 4) v = p->n_score;
+                else v = p->sub[4 * a + code];
+                c->dp.sv[5 * code + a] = v + oe;
+            }
         c->dp.one = 1;
         c->dp.zero = 0;
         c->dp.options = p->options;
@@ -330,8 +352,9 @@ int fastz_create(const fastz_params* p, const char* target, int64_t tlen, const 
     c->dp.eager_max = p->eager_max;
     c->tlen = (int)tlen;
     c->qlen = (int)qlen;
-    if ((r = upload_seq(c, target, tlen, c->Tf, c->Tr, 0, 0)) ||
-        (r = upload_seq(c, query, qlen, c->Qf, c->Qr, tlen, (p->options & FASTZ_OPT_QUERY_REVCOMP) ? 1 : 0))) {
+    if ((r = upload_seq(c, target, tlen, c->Tf, c->Tr, c->TfN, c->TrN, c->t_has_n, 0, 0)) ||
+        (r = upload_seq(c, query, qlen, c->Qf, c->Qr, c->QfN, c->QrN, c->q_has_n, tlen,
+                        (p->options & FASTZ_OPT_QUERY_REVCOMP) ? 1 : 0))) {
         fastz_destroy(c);
         return r;
     }
@@ -616,6 +639,7 @@ int fastz_find_hsps(fastz_ctx* c, const fastz_seed_params* spp, fastz_hsp* hsps,
     for (size_t i = 0; i < L; ++i) {
         if (spp->pattern[i] == '1') {
             if (sp.w == 16) return fail(FASTZ_EINVAL, "seed pattern has more than 16 care positions");
+            sp.caremask |= 1u << i;
             sp.off[sp.w++] = (int)i;
         } else if (spp->pattern[i] != '0') {
             return fail(FASTZ_EINVAL, "seed pattern characters must be '0' or '1'");
@@ -626,7 +650,8 @@ int fastz_find_hsps(fastz_ctx* c, const fastz_seed_params* spp, fastz_hsp* hsps,
     if (spp->xdrop < 0) return fail(FASTZ_EINVAL, "xdrop must be >= 0");
     sp.L = (int)L;
     UngappedParams up{};
-    for (int k = 0; k < 16; ++k) up.sub[k] = c->prm.sub[k];
+    for (int a = 0; a < 5; ++a)
+        for (int b = 0; b < 5; ++b) up.sub[5 * a + b] = (a == 4 || b == 4) ? c->prm.n_score : c->prm.sub[4 * a + b];
     up.xdrop = spp->xdrop;
     up.hspthresh = spp->hspthresh;
     const int nvar = spp->transitions ? 1 + sp.w : 1;
@@ -650,19 +675,37 @@ int fastz_find_hsps(fastz_ctx* c, const fastz_seed_params* spp, fastz_hsp* hsps,
     if (dense) AL(s_start, 4 * (nkeys + 1));
     AL(s_cnt, 8 * (QC + 1));
     AL(s_off, 8 * (QC + 1));
-    CK(seed_keys(P_<uint32_t>(c->Tf), nt, sp, P_<uint32_t>(c->s_kin), P_<int>(c->s_pin), st));
+    const uint16_t* TfN = c->t_has_n ? P_<uint16_t>(c->TfN) : nullptr;
+    const uint16_t* QfN = c->q_has_n ? P_<uint16_t>(c->QfN) : nullptr;
+    long long ntv = nt;  // target words in the index (S7: words with an N at a care position are dropped)
+    if (TfN) {
+        AL(s_keep, nt + 1);
+        AL(s_flag, 4);
+        CK(seed_keys(P_<uint32_t>(c->Tf), TfN, nt, sp, P_<uint32_t>(c->s_kout), P_<int>(c->s_pout),
+                     P_<unsigned char>(c->s_keep), st));
+        if (nt > 0) {
+            CK(seed_compact(c->s_tmp.p, tmpb, P_<uint32_t>(c->s_kout), P_<int>(c->s_pout), P_<unsigned char>(c->s_keep),
+                            nt, P_<uint32_t>(c->s_kin), P_<int>(c->s_pin), P_<int>(c->s_flag), st));
+            int nv = 0;
+            CK(cudaMemcpyAsync(&nv, c->s_flag.p, sizeof(int), cudaMemcpyDeviceToHost, st));
+            CK(cudaStreamSynchronize(st));
+            ntv = nv;
+        }
+    } else {
+        CK(seed_keys(P_<uint32_t>(c->Tf), nullptr, nt, sp, P_<uint32_t>(c->s_kin), P_<int>(c->s_pin), nullptr, st));
+    }
     CK(seed_sort_words(c->s_tmp.p, tmpb, P_<uint32_t>(c->s_kin), P_<uint32_t>(c->s_kout), P_<int>(c->s_pin),
-                       P_<int>(c->s_pout), nt, 2 * sp.w, st));
+                       P_<int>(c->s_pout), ntv, 2 * sp.w, st));
     const int* start = nullptr;
     if (dense) {
-        CK(seed_bucket_start(P_<uint32_t>(c->s_kout), nt, P_<int>(c->s_start), nkeys, st));
+        CK(seed_bucket_start(P_<uint32_t>(c->s_kout), ntv, P_<int>(c->s_start), nkeys, st));
         start = P_<int>(c->s_start);
     }
     // query chunks: count -> scan -> (D2H total) -> write hits -> ungapped walks -> select survivors
     long long q0 = 0, hits_total = 0, nlist = 0, list_cap = 0;
     while (q0 < nq) {
         const long long nqc = std::min(QC, nq - q0);
-        CK(seed_count(P_<uint32_t>(c->Qf), q0, nqc, sp, nvar, P_<uint32_t>(c->s_kout), P_<int>(c->s_pout), start, nt,
+        CK(seed_count(P_<uint32_t>(c->Qf), QfN, q0, nqc, sp, nvar, P_<uint32_t>(c->s_kout), P_<int>(c->s_pout), start, ntv,
                       P_<long long>(c->s_cnt), P_<long long>(c->s_off), c->s_tmp.p, tmpb, st));
         long long nh = 0;
         CK(cudaMemcpyAsync(&nh, P_<long long>(c->s_off) + nqc, sizeof(nh), cudaMemcpyDeviceToHost, st));
@@ -679,8 +722,8 @@ int fastz_find_hsps(fastz_ctx* c, const fastz_seed_params* spp, fastz_hsp* hsps,
             AL(s_sel, 16 * nh + 16);
             const size_t tb2 = seed_sort_tmp_bytes(nh);
             if (tb2 > c->s_tmp.cap) AL(s_tmp, tb2);
-            CK(seed_write_extend(P_<uint32_t>(c->Tf), P_<uint32_t>(c->Qf), c->tlen, c->qlen, q0, nqc, sp, nvar,
-                                 P_<uint32_t>(c->s_kout), P_<int>(c->s_pout), start, nt, P_<long long>(c->s_off), nh,
+            CK(seed_write_extend(P_<uint32_t>(c->Tf), P_<uint32_t>(c->Qf), TfN, QfN, c->tlen, c->qlen, q0, nqc, sp, nvar,
+                                 P_<uint32_t>(c->s_kout), P_<int>(c->s_pout), start, ntv, P_<long long>(c->s_off), nh,
                                  P_<int2>(c->s_hits), up, P_<int4>(c->s_hsp), P_<unsigned char>(c->s_keep), st));
             int* nsel_d = reinterpret_cast<int*>(P_<int4>(c->s_sel) + nh);
             CK(seed_select(c->s_tmp.p, c->s_tmp.cap, P_<int4>(c->s_hsp), P_<unsigned char>(c->s_keep), nh,

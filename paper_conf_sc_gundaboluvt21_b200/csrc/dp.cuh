@@ -32,20 +32,30 @@ constexpr unsigned FULL = 0xffffffffu;
 constexpr int SCORE_LIMIT = 1 << 29;
 constexpr int CP_RING = 128;      // column-profile ring entries per warp (+BLK mirrored)
 constexpr int EAGER_W = 17;       // eager code window: rows/cols 0..16 (16x16)
-// Substitution table in shared memory: entry e = code * 16 + a0 * 4 + a1 (query code 0..4, target bases of a
-// row pair) holds int2 {sub(a0, code) + O + E, sub(a1, code) + O + E} (code 4 = the origin column: sub = 0),
-// replicated 16x so that the 16 lanes of a half-warp read 16 distinct bank pairs (conflict-free LDS.64).
+// Substitution table in shared memory: entry e = code * NB^2 + a0 * NB + a1 (query code: A C G T = 0..3, 4 = the
+// origin column (sub = 0), 5 = N; target bases of a row pair a0, a1, 4 = N) holds int2
+// {sub(a0, code) + O + E, sub(a1, code) + O + E}, replicated 16x so that the 16 lanes of a half-warp read 16
+// distinct bank pairs (conflict-free LDS.64).  NB = 4 (codes 0..4) for batches without N -- the layout and
+// instruction stream of the N-free path are unchanged -- and NB = 5 (codes 0..5) when a sequence has an N
+// (reading R13: any pair with an N scores n_score).
 constexpr int SUBTAB_REP = 16;
 constexpr int SUBTAB_ENTRY = SUBTAB_REP * 8;    // bytes per entry
-constexpr int SUBTAB_CODE = 16 * SUBTAB_ENTRY;  // bytes per query code
-constexpr int SUBTAB_INTS = 5 * SUBTAB_CODE / 4;
+template <bool NM>
+struct SubTab {
+    static constexpr int NB = NM ? 5 : 4;                  // target-base symbols per row
+    static constexpr int CODE = NB * NB * SUBTAB_ENTRY;    // bytes per query code
+    static constexpr int NCODES = NM ? 6 : 5;
+    static constexpr int INTS = NCODES * CODE / 4;
+};
+constexpr int SUBTAB_INTS = SubTab<true>::INTS;  // shared allocation (the larger layout)
 
 // side flags
 constexpr uint32_t SF_EAGER = 1u, SF_OVERFLOW = 2u, SF_RING = 4u, SF_ESCALATE = 8u, SF_NOTB = 16u;
 constexpr int OPT_NO_EAGER = 1, OPT_NO_TRIM = 2, OPT_NO_BINNING = 4, OPT_NO_BLOCK = 8, OPT_TB_ABOVE_K = 16;
 
 struct DevParams {
-    int sv[20];        // sv[4b + a] = sub(a, b) + O + E for query base b = 0..3; sv[16 + a] = O + E (origin column)
+    int sv[30];        // sv[5 * code + a] = score(a, code) + O + E: code 0..3 query base, 4 origin column (0), 5 N;
+                       // target base a 0..3, 4 = N (reading R13: any pair with an N scores n_score)
     int O, E, Y, OE;   // gap open, extend, y-drop, O+E
     int K, eager_max;
     int one, zero;     // runtime 1 and 0: keep adds/selects as IMAD on the FMA pipe (ALU pipe is the limiter)
@@ -110,6 +120,11 @@ __device__ __forceinline__ int prmt(int a, int b, int s) {
 // base k (0-based position pos) of a 2-bit packed sequence (16 bases per word, base 0 in bits 1:0)
 __device__ __forceinline__ int base_at(const uint32_t* __restrict__ pk, int64_t pos) {
     return (int)((__ldg(pk + (pos >> 4)) >> ((pos & 15) * 2)) & 3u);
+}
+
+// N mask: bit (pos & 15) of 16-bit word pos >> 4 (nullptr: the sequence has no N)
+__device__ __forceinline__ bool n_at(const uint16_t* __restrict__ nm, int64_t pos) {
+    return nm != nullptr && ((__ldg(nm + (pos >> 4)) >> (pos & 15)) & 1u);
 }
 
 __device__ __forceinline__ int imax(int a, int b) { return a > b ? a : b; }

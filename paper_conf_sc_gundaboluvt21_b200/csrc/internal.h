@@ -22,6 +22,7 @@ struct SideArrays {
 
 struct Batch {
     const uint32_t *Tf, *Tr, *Qf, *Qr;  // packed target/query, forward and reversed
+    const uint16_t *TfN, *TrN, *QfN, *QrN;  // their N masks (nullptr when the sequence has no N)
     int tlen, qlen;
     const long long* seeds;             // (tpos, qpos) pairs
     int nseeds;
@@ -56,8 +57,8 @@ struct Outputs {
 
 int pick_R();  // rows per lane (FASTZ_R env: 2, 4 or 8; default 4)
 
-cudaError_t launch_pack(const char* src, int64_t n, uint32_t* fwd, uint32_t* rev, long long* bad, int revcomp,
-                        cudaStream_t st);
+cudaError_t launch_pack(const char* src, int64_t n, uint32_t* fwd, uint32_t* rev, uint16_t* fwdn, uint16_t* revn,
+                        long long* bad, int revcomp, cudaStream_t st);
 cudaError_t launch_validate_seeds(const long long* seeds, int n, int tlen, int qlen, long long* bad,
                                   cudaStream_t st);
 int inspector_blocks_per_sm(int R);
@@ -90,9 +91,10 @@ cudaError_t int_peak_run(int device, float ms, double* ops_per_s, double* mhz);
 struct SeedPattern {
     int L, w;      // span, care positions (1..16)
     int off[16];   // care offsets, ascending
+    unsigned caremask;  // bit o set for every care offset o
 };
 struct UngappedParams {
-    int sub[16];   // sub[4a+b], a = target base, b = query base
+    int sub[25];   // sub[5a+b], a = target code, b = query code, 4 = N (reading R13: n_score)
     int xdrop, hspthresh;
 };
 struct HspOut {    // layout of fastz_hsp
@@ -100,15 +102,17 @@ struct HspOut {    // layout of fastz_hsp
     int length, score;
 };
 size_t seed_sort_tmp_bytes(long long n);
-cudaError_t seed_keys(const uint32_t* Tf, long long nt, const SeedPattern& sp, uint32_t* keys, int* pos,
-                      cudaStream_t st);
+cudaError_t seed_keys(const uint32_t* Tf, const uint16_t* TfN, long long nt, const SeedPattern& sp, uint32_t* keys,
+                      int* pos, unsigned char* valid, cudaStream_t st);
+cudaError_t seed_compact(void* tmp, size_t tmp_bytes, const uint32_t* kin, const int* pin, const unsigned char* valid,
+                         long long nt, uint32_t* kout, int* pout, int* nsel, cudaStream_t st);
 cudaError_t seed_sort_words(void* tmp, size_t tmp_bytes, const uint32_t* kin, uint32_t* kout, const int* vin,
                             int* vout, long long n, int bits, cudaStream_t st);
 cudaError_t seed_bucket_start(const uint32_t* skeys, long long nt, int* start, long long nkeys, cudaStream_t st);
-cudaError_t seed_count(const uint32_t* Qf, long long q0, long long nq, const SeedPattern& sp, int nvar,
+cudaError_t seed_count(const uint32_t* Qf, const uint16_t* QfN, long long q0, long long nq, const SeedPattern& sp, int nvar,
                        const uint32_t* skeys, const int* spos, const int* start, long long nt, long long* cnt,
                        long long* off, void* tmp, size_t tmp_bytes, cudaStream_t st);
-cudaError_t seed_write_extend(const uint32_t* Tf, const uint32_t* Qf, int tlen, int qlen, long long q0, long long nq,
+cudaError_t seed_write_extend(const uint32_t* Tf, const uint32_t* Qf, const uint16_t* TfN, const uint16_t* QfN, int tlen, int qlen, long long q0, long long nq,
                               const SeedPattern& sp, int nvar, const uint32_t* skeys, const int* spos,
                               const int* start, long long nt, const long long* off, long long nh, int2* hits,
                               const UngappedParams& up, int4* hsp, unsigned char* keep, cudaStream_t st);

@@ -17,19 +17,21 @@ __device__ __forceinline__ int code_of(unsigned char c) {
         case 'C': case 'c': return 1;
         case 'G': case 'g': return 2;
         case 'T': case 't': return 3;
+        case 'N': case 'n': return 4;  // reading R13: packed as 0 plus a bit in the N mask
         default: return -1;
     }
 }
 
 __global__ void k_pack(const char* __restrict__ src, long long n, uint32_t* __restrict__ fwd,
-                       uint32_t* __restrict__ rev, long long* bad, int revcomp) {
+                       uint32_t* __restrict__ rev, uint16_t* __restrict__ fwdn, uint16_t* __restrict__ revn,
+                       long long* bad, int revcomp) {
     const long long w = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     const long long nw = (n + 15) / 16;
     if (w >= nw) return;
-    // revcomp: the sequence is the reverse complement of src (A<->T, C<->G: code xor 3), so its forward copy
-    // reads src backwards and its reversed copy reads src forwards, both complemented
+    // revcomp: the sequence is the reverse complement of src (A<->T, C<->G: code xor 3; N stays N), so its
+    // forward copy reads src backwards and its reversed copy reads src forwards, both complemented
     const uint32_t cx = revcomp ? 3u : 0u;
-    uint32_t f = 0, r = 0;
+    uint32_t f = 0, r = 0, fn = 0, rn = 0;
 #pragma unroll 4
     for (int i = 0; i < 16; ++i) {
         const long long p = 16 * w + i;
@@ -37,21 +39,26 @@ __global__ void k_pack(const char* __restrict__ src, long long n, uint32_t* __re
             const long long pf = revcomp ? n - 1 - p : p;
             int c = code_of((unsigned char)src[pf]);
             if (c < 0) { atomicMin(bad, pf); c = 0; }
+            if (c == 4) { fn |= 1u << i; c = 0; }
             f |= ((uint32_t)c ^ cx) << (2 * i);
             int cr = code_of((unsigned char)src[revcomp ? p : n - 1 - p]);
             if (cr < 0) cr = 0;
+            if (cr == 4) { rn |= 1u << i; cr = 0; }
             r |= ((uint32_t)cr ^ cx) << (2 * i);
         }
     }
     fwd[w] = f;
     rev[w] = r;
+    fwdn[w] = (uint16_t)fn;
+    revn[w] = (uint16_t)rn;
+    if (fn) atomicOr((unsigned long long*)(bad + 1), 1ull);  // the sequence has an N
 }
 
-cudaError_t launch_pack(const char* src, int64_t n, uint32_t* fwd, uint32_t* rev, long long* bad, int revcomp,
-                        cudaStream_t st) {
+cudaError_t launch_pack(const char* src, int64_t n, uint32_t* fwd, uint32_t* rev, uint16_t* fwdn, uint16_t* revn,
+                        long long* bad, int revcomp, cudaStream_t st) {
     const long long nw = (n + 15) / 16;
     if (nw == 0) return cudaSuccess;
-    k_pack<<<(unsigned)((nw + 255) / 256), 256, 0, st>>>(src, n, fwd, rev, bad, revcomp);
+    k_pack<<<(unsigned)((nw + 255) / 256), 256, 0, st>>>(src, n, fwd, rev, fwdn, revn, bad, revcomp);
     return cudaGetLastError();
 }
 
@@ -72,6 +79,7 @@ cudaError_t launch_validate_seeds(const long long* seeds, int n, int tlen, int q
 // ------------------------------------------------------------------------------------------------- sides
 // Side 2s is seed s's left extension (A_k = T[tpos-k], B_k = Q[qpos-k]: reversed copies starting at
 // tlen - tpos, qlen - qpos), side 2s+1 its right extension (A_k = T[tpos+k-1], B_k = Q[qpos+k-1]) -- P:168.
+template <bool NM>
 __device__ __forceinline__ void setup_side(const Batch& b, int side, SideIO& io) {
     const int seed = side >> 1;
     const long long tpos = b.seeds[2 * seed], qpos = b.seeds[2 * seed + 1];
@@ -81,6 +89,12 @@ __device__ __forceinline__ void setup_side(const Batch& b, int side, SideIO& io)
     } else {
         io.Apk = b.Tr; io.Aoff = b.tlen - tpos; io.M = (int)tpos;
         io.Bpk = b.Qr; io.Boff = b.qlen - qpos; io.Bmax = (int)qpos;
+    }
+    if constexpr (NM) {
+        __syncwarp();  // the previous side's last mask reads are done
+        io.ws->anm = (side & 1) ? b.TfN : b.TrN;
+        io.ws->bnm = (side & 1) ? b.QfN : b.QrN;
+        __syncwarp();
     }
     io.N = io.Bmax;
 }
@@ -93,16 +107,18 @@ struct SmemDP {
     uint8_t ecodes[WARPS][EAGER_W * EAGER_W + 15];
 };
 
+template <bool NM>
 __device__ __forceinline__ void smem_init(SmemDP& sm, const DevParams& P) {
-    for (int idx = threadIdx.x; idx < SUBTAB_INTS / 2; idx += blockDim.x) {
-        const int e = idx / SUBTAB_REP, code = e >> 4, a0 = (e >> 2) & 3, a1 = e & 3;
-        sm.subtab[2 * idx] = P.sv[4 * code + a0];
-        sm.subtab[2 * idx + 1] = P.sv[4 * code + a1];
+    using T = SubTab<NM>;
+    for (int idx = threadIdx.x; idx < T::INTS / 2; idx += blockDim.x) {
+        const int e = idx / SUBTAB_REP, code = e / (T::NB * T::NB), a0 = (e / T::NB) % T::NB, a1 = e % T::NB;
+        sm.subtab[2 * idx] = P.sv[5 * code + a0];
+        sm.subtab[2 * idx + 1] = P.sv[5 * code + a1];
     }
     // the column-code ring is read ahead of the strip's first column during ramp-up (dead cells): it must
     // always hold valid table offsets
     for (int idx = threadIdx.x; idx < WARPS * (CP_RING + BLK); idx += blockDim.x)
-        sm.w[idx / (CP_RING + BLK)].co[idx % (CP_RING + BLK)] = 4 * SUBTAB_CODE;
+        sm.w[idx / (CP_RING + BLK)].co[idx % (CP_RING + BLK)] = 4 * T::CODE;
     __syncthreads();
 }
 
@@ -166,24 +182,21 @@ __device__ __forceinline__ void write_side(const DevParams& P, const SideArrays&
     sa.nstrip[side] = notrim ? o.nstrips : -1;
 }
 
-// register budget of the inspector: by default only the CTA size is declared (ptxas then lands at 72
-// registers = 7 CTAs per SM, measured fastest); -DINSPECT_MIN_BLOCKS=n forces n resident CTAs per SM.  (An
-// explicit minimum of 1 is NOT the same: ptxas then spends 122 registers and occupancy drops to 4 CTAs.)
-#ifdef INSPECT_MIN_BLOCKS
-#define INSPECT_BOUNDS __launch_bounds__(WARPS * 32, INSPECT_MIN_BLOCKS)
-#else
-#define INSPECT_BOUNDS __launch_bounds__(WARPS * 32)
-#endif
+// register budget of the inspector: 72 registers = 7 resident CTAs of 4 warps per SM measured fastest.  ptxas's
+// own choice is fragile (72 or 115-122 registers for near-identical code, the latter at 4 CTAs per SM and ~20%
+// slower): the N-free instantiation lands at 72 by itself (an explicit cap there costs 3 instructions per step),
+// the N-aware one (k_inspect_n) is capped with __maxnreg__ (any explicit attribute on the N-free kernel, even
+// __maxnreg__(255) or a minimum of 1 CTA, moves it to ~120 registers).
 // ------------------------------------------------------------------------------------------------- inspector
 // Persistent: each warp pops one-sided extensions from an atomic queue (load balance replaces the paper's
 // 32 CUDA streams).  Score-only DP + eager 17x17 corner codes; when the peak lies inside the
 // eager window the warp's lane 0 walks the codes at once and the side skips the executor.
 // A side still running after `budget` strips is handed to the block-per-side inspector (escalation).
-template <int R>
-__global__ void INSPECT_BOUNDS k_inspect(DevParams P, Batch b, int4* ring, int rmask,
-                                                         SideArrays sa, ExecPlan pl, int budget) {
+template <int R, bool NM>
+__device__ __forceinline__ void inspect_body(const DevParams& P, const Batch& b, int4* ring, int rmask,
+                                             const SideArrays& sa, const ExecPlan& pl, int budget) {
     __shared__ SmemDP sm;
-    smem_init(sm, P);
+    smem_init<NM>(sm, P);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     SideIO io;
     io_init(io, sm, ring, rmask, blockIdx.x * WARPS + warp, warp);
@@ -195,9 +208,9 @@ __global__ void INSPECT_BOUNDS k_inspect(DevParams P, Batch b, int4* ring, int r
         if (lane == 0) side = atomicAdd(&pl.counters[0], 1);
         side = __shfl_sync(FULL, side, 0);
         if (side >= nsides) break;
-        setup_side(b, side, io);
+        setup_side<NM>(b, side, io);
         SideOut o;
-        run_side<R, MODE_INSPECT, true, false>(P, io, o);
+        run_side<R, MODE_INSPECT, true, false, NM>(P, io, o);
         __syncwarp();  // eager corner codes (shared memory) written by lanes 0..4 -> read by lane 0
         if (lane == 0) {
             if (o.flags & SF_ESCALATE) {
@@ -218,14 +231,25 @@ __global__ void INSPECT_BOUNDS k_inspect(DevParams P, Batch b, int4* ring, int r
     }
 }
 
-// Block per side (long sides, escalated by k_inspect): the CTA's warps pipeline the side's strips.
 template <int R>
+__global__ void __launch_bounds__(WARPS * 32) k_inspect(DevParams P, Batch b, int4* ring, int rmask, SideArrays sa,
+                                                         ExecPlan pl, int budget) {
+    inspect_body<R, false>(P, b, ring, rmask, sa, pl, budget);
+}
+template <int R>
+__global__ void __maxnreg__(72) k_inspect_n(DevParams P, Batch b, int4* ring, int rmask,
+                                                                           SideArrays sa, ExecPlan pl, int budget) {
+    inspect_body<R, true>(P, b, ring, rmask, sa, pl, budget);
+}
+
+// Block per side (long sides, escalated by k_inspect): the CTA's warps pipeline the side's strips.
+template <int R, bool NM>
 __global__ void __launch_bounds__(WARPS * 32) k_inspect_block(DevParams P, Batch b, int4* ring, int rmask,
                                                                SideArrays sa, ExecPlan pl) {
     __shared__ SmemDP sm;
     __shared__ PipeShared ps;
     __shared__ int cur;
-    smem_init(sm, P);
+    smem_init<NM>(sm, P);
     const int warp = threadIdx.x >> 5;
     for (;;) {
         if (threadIdx.x == 0) {
@@ -239,19 +263,19 @@ __global__ void __launch_bounds__(WARPS * 32) k_inspect_block(DevParams P, Batch
         SideIO io;
         io_init(io, sm, ring, rmask, blockIdx.x * WARPS, warp);
         io.ps = &ps;
-        setup_side(b, side, io);
+        setup_side<NM>(b, side, io);
         SideOut o;
-        run_side<R, MODE_INSPECT, false, true>(P, io, o);
+        run_side<R, MODE_INSPECT, false, true, NM>(P, io, o);
         if (threadIdx.x == 0) write_side(P, sa, side, o, o.flags, 0ull, 0);
         __syncthreads();
     }
 }
 
-template <int R>
+template <int R, bool NM>
 __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int4* ring, int rmask,
                                                         long long* cells, int* counter) {
     __shared__ SmemDP sm;
-    smem_init(sm, P);
+    smem_init<NM>(sm, P);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     SideIO io;
     io_init(io, sm, ring, rmask, blockIdx.x * WARPS + warp, warp);
@@ -261,9 +285,9 @@ __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int
         if (lane == 0) side = atomicAdd(counter, 1);
         side = __shfl_sync(FULL, side, 0);
         if (side >= nsides) break;
-        setup_side(b, side, io);
+        setup_side<NM>(b, side, io);
         SideOut o;
-        run_side<R, MODE_CENSUS, false, false>(P, io, o);
+        run_side<R, MODE_CENSUS, false, false, NM>(P, io, o);
         if (lane == 0) cells[side] = (o.flags & SF_RING) ? -1 : o.cells;
         __syncwarp();
     }
@@ -273,14 +297,14 @@ __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int
 // Trimmed executor: the DP over [0,i*]x[0,j*] only, writing traceback codes.  Length binning
 // as a schedule: the CTAs first take the long sides (bins >= 3, block per side, strips pipelined
 // across the CTA's warps), then every warp takes short sides (bins 1-2, warp per side), larger bins first.
-template <int R>
+template <int R, bool NM>
 __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, int4* ring, int rmask,
                                                          SideArrays sa, ExecPlan pl, int lo, int hi, int nblock,
                                                          long long base, Outputs out) {
     __shared__ SmemDP sm;
     __shared__ PipeShared ps;
     __shared__ int cur;
-    smem_init(sm, P);
+    smem_init<NM>(sm, P);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     for (;;) {  // block phase
         if (threadIdx.x == 0) {
@@ -294,7 +318,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, in
         SideIO io;
         io_init(io, sm, ring, rmask, blockIdx.x * WARPS, warp);
         io.ps = &ps;
-        setup_side(b, side, io);
+        setup_side<NM>(b, side, io);
         if (!(P.options & OPT_NO_TRIM)) {  // trimmed executor: the rectangle up to the peak
             io.M = sa.ti[side];
             io.N = sa.qj[side];
@@ -303,7 +327,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, in
         io.stab = out.stab + pl.soff[side];
         io.maxsw = sa.maxsw[side];
         SideOut o;
-        run_side<R, MODE_EXEC, false, true>(P, io, o);
+        run_side<R, MODE_EXEC, false, true, NM>(P, io, o);
         if (threadIdx.x == 0 && (o.flags & SF_RING)) atomicOr(&sa.flags[side], SF_RING);
         __syncthreads();
     }
@@ -315,7 +339,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, in
         idx = __shfl_sync(FULL, idx, 0);
         if (idx >= hi) break;
         const int side = pl.list[idx];
-        setup_side(b, side, io);
+        setup_side<NM>(b, side, io);
         if (!(P.options & OPT_NO_TRIM)) {
             io.M = sa.ti[side];
             io.N = sa.qj[side];
@@ -323,7 +347,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, in
         io.codes = out.codes + (pl.woff[side] - base);
         io.stab = out.stab + pl.soff[side];
         SideOut o;
-        run_side<R, MODE_EXEC, false, false>(P, io, o);
+        run_side<R, MODE_EXEC, false, false, NM>(P, io, o);
         if (lane == 0 && (o.flags & SF_RING)) atomicOr(&sa.flags[side], SF_RING);
         __syncwarp();
     }
@@ -519,9 +543,10 @@ __global__ void k_bin_offsets(ExecPlan pl, int nsides, const long long* words, c
 }
 
 // pool offsets in executor (list) order, so that a wave is a contiguous range of the list
-__global__ void k_list_words(ExecPlan pl, const long long* words, long long* wl) {
+__global__ void k_list_words(ExecPlan pl, const long long* words, long long* wl, int nsides) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
-    if (i < (int)pl.totals[3]) wl[i] = words[pl.list[i]];
+    // positions past the executor list are scanned too (the scan runs over nsides): define them as 0
+    if (i < nsides) wl[i] = i < (int)pl.totals[3] ? words[pl.list[i]] : 0;
 }
 __global__ void k_list_offsets(ExecPlan pl, const long long* wlo, const long long* wl) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
@@ -570,7 +595,7 @@ cudaError_t launch_bin(int R, const DevParams& P, const SideArrays& sa, int nsid
         k_bin_scatter<<<g, 256, 0, st>>>(pl, nsides);
         long long* wl = pl.wl;
         long long* wlo = pl.wlo;
-        k_list_words<<<g, 256, 0, st>>>(pl, words, wl);
+        k_list_words<<<g, 256, 0, st>>>(pl, words, wl, nsides);
         size_t b = tmp_bytes;
         if ((e = cub::DeviceScan::ExclusiveSum(tmp, b, wl, wlo, nsides, st)) != cudaSuccess) return e;
         k_list_offsets<<<g, 256, 0, st>>>(pl, wlo, wl);
@@ -726,8 +751,14 @@ int inspector_blocks_per_sm(int R) { return R == 2 ? bps_of<2>() : bps_of<4>(); 
 
 #define FZ_DISPATCH(KERNEL, GRID, ...)                                                   \
     do {                                                                                 \
-        if (R == 2) KERNEL<2><<<GRID, WARPS * 32, 0, st>>>(__VA_ARGS__);                 \
-        else KERNEL<4><<<GRID, WARPS * 32, 0, st>>>(__VA_ARGS__);                        \
+        const bool nm_ = b.TfN || b.QfN; /* N masks present: the N-aware instantiation */ \
+        if (R == 2) {                                                                    \
+            if (nm_) KERNEL<2, true><<<GRID, WARPS * 32, 0, st>>>(__VA_ARGS__);          \
+            else KERNEL<2, false><<<GRID, WARPS * 32, 0, st>>>(__VA_ARGS__);             \
+        } else {                                                                         \
+            if (nm_) KERNEL<4, true><<<GRID, WARPS * 32, 0, st>>>(__VA_ARGS__);          \
+            else KERNEL<4, false><<<GRID, WARPS * 32, 0, st>>>(__VA_ARGS__);             \
+        }                                                                                \
     } while (0)
 
 // Inspector escalation of long sides to the block-per-side inspector (FASTZ_ESCALATE_STRIPS, strips; 0 = off).
@@ -746,7 +777,14 @@ int escalate_strips() {  // read per call: tests and ablations switch it at run 
 cudaError_t launch_inspect(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
                            const SideArrays& sa, const ExecPlan& pl, int budget, cudaStream_t st) {
     if (b.nseeds == 0) return cudaSuccess;
-    FZ_DISPATCH(k_inspect, grid, P, b, ring, rmask, sa, pl, budget);
+    const bool nm = b.TfN || b.QfN;
+    if (R == 2) {
+        if (nm) k_inspect_n<2><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, pl, budget);
+        else k_inspect<2><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, pl, budget);
+    } else {
+        if (nm) k_inspect_n<4><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, pl, budget);
+        else k_inspect<4><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, pl, budget);
+    }
     return cudaGetLastError();
 }
 

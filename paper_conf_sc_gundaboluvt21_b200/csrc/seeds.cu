@@ -43,12 +43,22 @@ __device__ __forceinline__ uint32_t seed_word(const uint32_t* __restrict__ pk, l
     return k;
 }
 
-__global__ void k_seed_keys(const uint32_t* __restrict__ Tf, long long nt, SeedPattern sp, uint32_t* keys,
-                            int* pos) {
+// S7: does the word at position p have an N at a care position?  (nm == nullptr: the sequence has no N)
+__device__ __forceinline__ bool care_has_n(const uint16_t* __restrict__ nm, long long p, const SeedPattern& sp) {
+    if (nm == nullptr) return false;
+    const long long w0 = p >> 4;
+    const unsigned long long bits = (unsigned long long)__ldg(nm + w0) | ((unsigned long long)__ldg(nm + w0 + 1) << 16) |
+                                    ((unsigned long long)__ldg(nm + w0 + 2) << 32);  // masks carry 4 pad words
+    return ((bits >> (p & 15)) & sp.caremask) != 0;
+}
+
+__global__ void k_seed_keys(const uint32_t* __restrict__ Tf, const uint16_t* __restrict__ TfN, long long nt,
+                            SeedPattern sp, uint32_t* keys, int* pos, unsigned char* valid) {
     const long long p = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     if (p >= nt) return;
     keys[p] = seed_word(Tf, p, sp);
     pos[p] = (int)p;
+    if (valid) valid[p] = care_has_n(TfN, p, sp) ? 0 : 1;
 }
 
 // dense bucket starts: start[k] = first sorted index with key >= k, k in [0, 4^w]
@@ -94,11 +104,11 @@ __device__ __forceinline__ uint32_t variant(uint32_t k0, int v, int w) {
     return v == 0 ? k0 : k0 ^ (2u << (2 * (w - v)));
 }
 
-__global__ void k_seed_count(const uint32_t* __restrict__ Qf, long long q0, long long nq, SeedPattern sp,
-                             int nvar, SeedIndex ix, long long* cnt) {
+__global__ void k_seed_count(const uint32_t* __restrict__ Qf, const uint16_t* __restrict__ QfN, long long q0,
+                             long long nq, SeedPattern sp, int nvar, SeedIndex ix, long long* cnt) {
     const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     if (i > nq) return;
-    if (i == nq) {
+    if (i == nq || care_has_n(QfN, q0 + i, sp)) {  // S7
         cnt[i] = 0;
         return;
     }
@@ -112,10 +122,11 @@ __global__ void k_seed_count(const uint32_t* __restrict__ Qf, long long q0, long
     cnt[i] = n;
 }
 
-__global__ void k_seed_write(const uint32_t* __restrict__ Qf, long long q0, long long nq, SeedPattern sp, int nvar,
-                             SeedIndex ix, const long long* __restrict__ off, int2* hits) {
+__global__ void k_seed_write(const uint32_t* __restrict__ Qf, const uint16_t* __restrict__ QfN, long long q0,
+                             long long nq, SeedPattern sp, int nvar, SeedIndex ix, const long long* __restrict__ off,
+                             int2* hits) {
     const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-    if (i >= nq) return;
+    if (i >= nq || care_has_n(QfN, q0 + i, sp)) return;  // S7
     const uint32_t k0 = seed_word(Qf, q0 + i, sp);
     long long o = off[i];
     for (int v = 0; v < nvar; ++v) {
@@ -125,32 +136,39 @@ __global__ void k_seed_write(const uint32_t* __restrict__ Qf, long long q0, long
     }
 }
 
-// Reads consecutive bases of a 2-bit packed sequence (either direction) with one load per 16 bases.
+// Reads consecutive bases of a 2-bit packed sequence (either direction) with one load per 16 bases; with an N
+// mask (nm != nullptr) an N reads as code 4.
 struct BaseStream {
     const uint32_t* pk;
+    const uint16_t* nm;
     long long word;
-    uint32_t cur;
-    __device__ __forceinline__ void init(const uint32_t* p, long long pos) {
+    uint32_t cur, curn;
+    __device__ __forceinline__ void init(const uint32_t* p, const uint16_t* m, long long pos) {
         pk = p;
+        nm = m;
         word = pos >> 4;
         cur = __ldg(pk + word);
+        curn = nm ? __ldg(nm + word) : 0u;
     }
     __device__ __forceinline__ int get(long long pos) {
         const long long w = pos >> 4;
         if (w != word) {
             word = w;
             cur = __ldg(pk + w);
+            curn = nm ? __ldg(nm + w) : 0u;
         }
-        return (int)((cur >> ((pos & 15) * 2)) & 3u);
+        const int sh = (int)(pos & 15);
+        return (int)((cur >> (sh * 2)) & 3u) | (int)(((curn >> sh) & 1u) << 2);
     }
 };
 
 // S3 + S4: one thread per hit.  out[h] = {t_start, q_start, length, score}; keep[h] = score >= thresh.
 __global__ void k_ungapped(const int2* __restrict__ hits, long long nh, const uint32_t* __restrict__ Tf,
-                           const uint32_t* __restrict__ Qf, int tlen, int qlen, UngappedParams up, int4* out,
+                           const uint32_t* __restrict__ Qf, const uint16_t* __restrict__ TfN,
+                           const uint16_t* __restrict__ QfN, int tlen, int qlen, UngappedParams up, int4* out,
                            unsigned char* keep) {
-    __shared__ int sub[16];
-    if (threadIdx.x < 16) sub[threadIdx.x] = up.sub[threadIdx.x];
+    __shared__ int sub[25];
+    if (threadIdx.x < 25) sub[threadIdx.x] = up.sub[threadIdx.x];
     __syncthreads();
     const long long h = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     if (h >= nh) return;
@@ -161,10 +179,10 @@ __global__ void k_ungapped(const int2* __restrict__ hits, long long nh, const ui
     int s = 0, best_r = 0, r = 0;
     const int nr = min(tlen - t, qlen - q);
     if (nr > 0) {
-        ts.init(Tf, t);
-        qs.init(Qf, q);
+        ts.init(Tf, TfN, t);
+        qs.init(Qf, QfN, q);
         for (int d = 0; d < nr; ++d) {
-            s += sub[4 * ts.get(t + d) + qs.get(q + d)];
+            s += sub[5 * ts.get(t + d) + qs.get(q + d)];
             if (s > best_r) {
                 best_r = s;
                 r = d + 1;
@@ -177,10 +195,10 @@ __global__ void k_ungapped(const int2* __restrict__ hits, long long nh, const ui
     s = 0;
     const int nl = min(t, q);
     if (nl > 0) {
-        ts.init(Tf, t - 1);
-        qs.init(Qf, q - 1);
+        ts.init(Tf, TfN, t - 1);
+        qs.init(Qf, QfN, q - 1);
         for (int d = 1; d <= nl; ++d) {
-            s += sub[4 * ts.get(t - d) + qs.get(q - d)];
+            s += sub[5 * ts.get(t - d) + qs.get(q - d)];
             if (s > best_l) {
                 best_l = s;
                 l = d;
@@ -244,11 +262,19 @@ __global__ void k_hsp_emit(const int4* __restrict__ hs, const int* __restrict__ 
 static inline unsigned nblk(long long n, int t = 256) { return (unsigned)((n + t - 1) / t); }
 
 // ------------------------------------------------------------------------------------------------ launchers
-cudaError_t seed_keys(const uint32_t* Tf, long long nt, const SeedPattern& sp, uint32_t* keys, int* pos,
-                      cudaStream_t st) {
+cudaError_t seed_keys(const uint32_t* Tf, const uint16_t* TfN, long long nt, const SeedPattern& sp, uint32_t* keys,
+                      int* pos, unsigned char* valid, cudaStream_t st) {
     if (nt <= 0) return cudaSuccess;
-    k_seed_keys<<<nblk(nt), 256, 0, st>>>(Tf, nt, sp, keys, pos);
+    k_seed_keys<<<nblk(nt), 256, 0, st>>>(Tf, TfN, nt, sp, keys, pos, valid);
     return cudaGetLastError();
+}
+
+// S7: drop target words with an N at a care position before the sort (two selects: words, positions)
+cudaError_t seed_compact(void* tmp, size_t tmp_bytes, const uint32_t* kin, const int* pin, const unsigned char* valid,
+                         long long nt, uint32_t* kout, int* pout, int* nsel, cudaStream_t st) {
+    cudaError_t e = cub::DeviceSelect::Flagged(tmp, tmp_bytes, kin, valid, kout, nsel, (int)nt, st);
+    if (e != cudaSuccess) return e;
+    return cub::DeviceSelect::Flagged(tmp, tmp_bytes, pin, valid, pout, nsel, (int)nt, st);
 }
 
 size_t seed_sort_tmp_bytes(long long n) {
@@ -260,9 +286,13 @@ size_t seed_sort_tmp_bytes(long long n) {
     cub::DeviceScan::ExclusiveSum(nullptr, c, (const long long*)nullptr, (long long*)nullptr, (int)(n > 0 ? n + 1 : 2));
     cub::DeviceSelect::Flagged(nullptr, d, (const int4*)nullptr, (const unsigned char*)nullptr, (int4*)nullptr,
                                (int*)nullptr, (int)(n > 0 ? n : 1));
-    size_t e = 0;
+    size_t e = 0, f = 0, g = 0;
     cub::DeviceScan::ExclusiveSum(nullptr, e, (const int*)nullptr, (int*)nullptr, (int)(n > 0 ? n + 1 : 2));
-    return std::max(std::max(std::max(a, b), std::max(c, d)), e);
+    cub::DeviceSelect::Flagged(nullptr, f, (const uint32_t*)nullptr, (const unsigned char*)nullptr, (uint32_t*)nullptr,
+                               (int*)nullptr, (int)(n > 0 ? n : 1));
+    cub::DeviceSelect::Flagged(nullptr, g, (const int*)nullptr, (const unsigned char*)nullptr, (int*)nullptr,
+                               (int*)nullptr, (int)(n > 0 ? n : 1));
+    return std::max(std::max(std::max(a, b), std::max(c, d)), std::max(e, std::max(f, g)));
 }
 
 cudaError_t seed_sort_words(void* tmp, size_t tmp_bytes, const uint32_t* kin, uint32_t* kout, const int* vin,
@@ -278,24 +308,25 @@ cudaError_t seed_bucket_start(const uint32_t* skeys, long long nt, int* start, l
     return cudaGetLastError();
 }
 
-cudaError_t seed_count(const uint32_t* Qf, long long q0, long long nq, const SeedPattern& sp, int nvar,
-                       const uint32_t* skeys, const int* spos, const int* start, long long nt, long long* cnt,
+cudaError_t seed_count(const uint32_t* Qf, const uint16_t* QfN, long long q0, long long nq, const SeedPattern& sp,
+                       int nvar, const uint32_t* skeys, const int* spos, const int* start, long long nt, long long* cnt,
                        long long* off, void* tmp, size_t tmp_bytes, cudaStream_t st) {
     SeedIndex ix{skeys, spos, start, nt};
-    k_seed_count<<<nblk(nq + 1), 256, 0, st>>>(Qf, q0, nq, sp, nvar, ix, cnt);
+    k_seed_count<<<nblk(nq + 1), 256, 0, st>>>(Qf, QfN, q0, nq, sp, nvar, ix, cnt);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
     return cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, cnt, off, (int)(nq + 1), st);
 }
 
-cudaError_t seed_write_extend(const uint32_t* Tf, const uint32_t* Qf, int tlen, int qlen, long long q0, long long nq,
+cudaError_t seed_write_extend(const uint32_t* Tf, const uint32_t* Qf, const uint16_t* TfN, const uint16_t* QfN, int tlen,
+                              int qlen, long long q0, long long nq,
                               const SeedPattern& sp, int nvar, const uint32_t* skeys, const int* spos,
                               const int* start, long long nt, const long long* off, long long nh, int2* hits,
                               const UngappedParams& up, int4* hsp, unsigned char* keep, cudaStream_t st) {
     if (nq <= 0 || nh <= 0) return cudaSuccess;
     SeedIndex ix{skeys, spos, start, nt};
-    k_seed_write<<<nblk(nq), 256, 0, st>>>(Qf, q0, nq, sp, nvar, ix, off, hits);
-    k_ungapped<<<nblk(nh), 256, 0, st>>>(hits, nh, Tf, Qf, tlen, qlen, up, hsp, keep);
+    k_seed_write<<<nblk(nq), 256, 0, st>>>(Qf, QfN, q0, nq, sp, nvar, ix, off, hits);
+    k_ungapped<<<nblk(nh), 256, 0, st>>>(hits, nh, Tf, Qf, TfN, QfN, tlen, qlen, up, hsp, keep);
     return cudaGetLastError();
 }
 

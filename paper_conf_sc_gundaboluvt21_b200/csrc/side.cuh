@@ -52,10 +52,14 @@ constexpr int BLK = 32;
 constexpr int PIPE_SLOTS = 8;  // 2K slots for K = 4 warps: a slot is reused only after its consumer finished
 
 struct WarpSmem {
-    int co[CP_RING + BLK];  // column codes of the query side as substitution-table byte offsets (code * SUBTAB_CODE),
+    int co[CP_RING + BLK];  // column codes of the query side as substitution-table byte offsets (code * SubTab::CODE),
                             // ring over relative columns (+BLK mirrored)
     int4 bin[BLK];          // boundary row staging {X, D, W, -}: lane 0's input of the current block
     int4 bout[BLK];         // lane 31's bottom-row outputs {X, D, W, -} awaiting the global ring
+    // N masks of the side's target / query copies (nullptr: no N); kept here rather than in registers so the
+    // strip loop's register budget (72 = 7 CTAs per SM) is unchanged -- read only at strip set-up and staging
+    const uint16_t* anm;
+    const uint16_t* bnm;
 };
 
 // Block-per-problem (PIPE) shared state of one side.  Strip s owns slot s % PIPE_SLOTS.
@@ -114,12 +118,20 @@ struct StripGeom {
     static constexpr int SPW = 8 / R;  // steps per 32-bit code word
 };
 
+// column code: query base 0..3, 5 for an N (NM: the batch has N masks), 4 outside [1, N] (the origin column and
+// beyond the end)
+template <bool NM>
 __device__ __forceinline__ int query_code(const SideIO& io, int c) {
-    return (c >= 1 && c <= io.N) ? base_at(io.Bpk, io.Boff + c - 1) : 4;
+    if (c < 1 || c > io.N) return 4;
+    if constexpr (NM) {
+        if (n_at(io.ws->bnm, io.Boff + c - 1)) return 5;
+    }
+    return base_at(io.Bpk, io.Boff + c - 1);
 }
 
+template <bool NM>
 __device__ __forceinline__ void cp_store(const SideIO& io, int rc, int code) {
-    const int v = code * SUBTAB_CODE;
+    const int v = code * SubTab<NM>::CODE;
     const int idx = rc & (CP_RING - 1);
     io.ws->co[idx] = v;
     if (idx < BLK) io.ws->co[idx + CP_RING] = v;
@@ -135,7 +147,7 @@ __device__ __forceinline__ int4 boundary(const int4* __restrict__ ring, int rmas
 
 __device__ __forceinline__ void pipe_wait() { __nanosleep(100); }
 
-template <int R, int MODE, bool EAGER, bool PIPE>
+template <int R, int MODE, bool EAGER, bool PIPE, bool NM>
 __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, SideOut& out) {
     constexpr int H = StripGeom<R>::H;
     constexpr int SPW = StripGeom<R>::SPW;
@@ -224,8 +236,8 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         for (int k = 0; k < R; ++k) {
             const int r = r0 + k;
             int a = 0;
-            if (r >= 1 && r <= M) a = base_at(io.Apk, io.Aoff + r - 1);
-            if (k % 2 == 0) tb[k / 2] = io.subtab + (unsigned)(a * 4 * SUBTAB_ENTRY) + (unsigned)((lane & 15) * 8);
+            if (r >= 1 && r <= M) a = (NM && n_at(io.ws->anm, io.Aoff + r - 1)) ? 4 : base_at(io.Apk, io.Aoff + r - 1);
+            if (k % 2 == 0) tb[k / 2] = io.subtab + (unsigned)(a * SubTab<NM>::NB * SUBTAB_ENTRY) + (unsigned)((lane & 15) * 8);
             else tb[k / 2] += (unsigned)(a * SUBTAB_ENTRY);
             X[k] = NEG;
             I[k] = NEG;
@@ -276,9 +288,9 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         int qpre = 4;
         if (stager) {
             ws->bin[lane] = boundary<PIPE>(ring, rmask, start + lane, blim, bwf);
-            cp_store(io, lane, query_code(io, start + lane));
+            cp_store<NM>(io, lane, query_code<NM>(io, start + lane));
             bpre = boundary<PIPE>(ring, rmask, start + BK + lane, blim, bwf);
-            qpre = query_code(io, start + BK + lane);
+            qpre = query_code<NM>(io, start + BK + lane);
         }
         __syncwarp();
         uint32_t cw = 0;
@@ -471,9 +483,9 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                 if (stager) {
                     const int rcn = t + lane;
                     ws->bin[rcn & (BK - 1)] = bpre;
-                    cp_store(io, rcn, qpre);
+                    cp_store<NM>(io, rcn, qpre);
                     bpre = boundary<PIPE>(ring, rmask, start + rcn + BK, blim, bwf);
-                    qpre = query_code(io, start + rcn + BK);
+                    qpre = query_code<NM>(io, start + rcn + BK);
                 }
             }
             __syncwarp();

@@ -37,7 +37,8 @@ class FastzError(RuntimeError):
 class fastz_params(ctypes.Structure):
     _fields_ = [("sub", ctypes.c_int32 * 16), ("gap_open", ctypes.c_int32), ("gap_extend", ctypes.c_int32),
                 ("ydrop", ctypes.c_int32), ("gapped_threshold", ctypes.c_int32), ("eager_max", ctypes.c_int32),
-                ("options", ctypes.c_int32), ("reserved", ctypes.c_int32 * 2), ("dev_alloc", ctypes.c_void_p),
+                ("options", ctypes.c_int32), ("n_score", ctypes.c_int32), ("reserved", ctypes.c_int32),
+                ("dev_alloc", ctypes.c_void_p),
                 ("dev_free", ctypes.c_void_p),
                 ("alloc_user", ctypes.c_void_p)]
 

@@ -78,7 +78,7 @@ def test_sass_targets_sm100a_and_uses_the_integer_dp_instructions():
     out = subprocess.check_output(["/usr/local/cuda/bin/cuobjdump", "-sass", build.build()]).decode()
     sections = out.split("Function : ")
     names = [sec.split("\n", 1)[0] for sec in sections[1:]]
-    for k in ("k_inspectILi4EE", "k_inspect_blockILi4EE", "k_executeILi4EE", "k_censusILi4EE",
+    for k in ("k_inspectILi4EE", "k_inspect_nILi4EE", "k_inspect_blockILi4E", "k_executeILi4E", "k_censusILi4E",
               "k_traceback", "k_pack", "k_bin_count", "k_combine_write"):
         assert any(k in n for n in names), k
     insp = next(sec for sec in sections[1:] if sec.startswith("_ZN2fz9k_inspectILi4EE"))

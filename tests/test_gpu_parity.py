@@ -236,3 +236,19 @@ def test_traceback_above_k_only():
             assert g1.cigar_of(s) == g0.cigar_of(s)
         else:
             assert g1.rec["cigar_len"][s] == 0 and g1.rec["flags"][s] & fz.FLAG_NO_CIGAR
+
+
+@pytest.mark.parametrize("n_score", [-100, 0, 60])
+def test_n_bases(n_score):
+    """N bases (reading R13: any pair with an N scores n_score) in both sequences, isolated and in runs, on a
+    mixed workload: bit-exact per seed and per side, explored-cell census included."""
+    rng = np.random.default_rng(500 + n_score)
+    w = genome.small_pair(21, length=20000, n_seeds=300)
+    def with_ns(s, k, run):
+        s = bytearray(s)
+        for p in rng.choice(len(s) - run, k, replace=False):
+            s[p:p + run] = b"N" * run
+        return bytes(s)
+    T = with_ns(with_ns(w.T, 200, 1), 5, 30)
+    Q = with_ns(with_ns(w.Q, 200, 1), 5, 30).lower()
+    assert_ok(compare(T, Q, w.seeds, census=True, n_score=n_score)[0])

@@ -100,4 +100,31 @@ def test_minus_strand():
     assert all(ga.cigar_of(s) == orr.cigar_of(s) for s in range(len(an)))
     # invalid character reported at its index in the caller's string
     with pytest.raises(fastz.FastzError, match="index"):
-        fastz.Aligner(T, Qm[:100] + "N" + Qm[101:], fastz.fastz_default_params(options=32))
+        fastz.Aligner(T, Qm[:100] + "X" + Qm[101:], fastz.fastz_default_params(options=32))
+
+
+def with_ns(s: str, rng, k: int, run: int = 1) -> str:
+    s = list(s)
+    for p in rng.choice(len(s) - run, k, replace=False):
+        for d in range(run):
+            s[p + d] = "N"
+    return "".join(s)
+
+
+@pytest.mark.parametrize("n_score", [-100, 0])
+def test_n_bases_seeding_and_pipeline(n_score):
+    """N (reading R13 / S7) on both sequences, both strands: HSPs equal the oracle's; anchors -> gapped parity."""
+    rng = np.random.default_rng(11)
+    w = genome.small_pair(9, length=30000, n_seeds=8)
+    T = with_ns(w.T.decode(), rng, 60) ; T = with_ns(T, rng, 3, run=40)
+    Q = with_ns(w.Q.decode(), rng, 60)
+    for opts, Qo in ((0, Q), (32, revcomp(Q))):
+        with fastz.Aligner(T, Q, fastz.fastz_default_params(options=opts, n_score=n_score)) as al:
+            g, an, gh = al.find_hsps()
+            ga = al.extend(an)
+        o, oh = seeds.find_hsps(T, Qo, core.HOXD70, n_score=n_score)
+        assert_same(g, an, gh, o, oh)
+        orr = core.extend(T, Qo, an, core.Params(n_score=n_score))
+        for f in ("score", "t_start", "t_end", "q_start", "q_end"):
+            assert np.array_equal(ga.rec[f].astype(np.int64), orr.rec[f]), f
+        assert all(ga.cigar_of(s) == orr.cigar_of(s) for s in range(len(an)))
