@@ -359,12 +359,14 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                     const int d = __viaddmax_s32(du, mE, xu);
                     const int iv = __viaddmax_s32(I[k], mE, X[k]);
                     const int sr = __vimax3_s32(h, d, iv);
-                    // W = max(thr, S_raw - Y) with thr = max(W_up, W_left): for a dead cell S_raw - Y < thr, so
-                    // this equals max(thr, S_live - Y) (reading R3), and since Y >= 0 the cell is live iff
-                    // S_raw >= W (S >= thr => W <= S; S < thr => W >= thr > S): the threshold max and the
-                    // live test share one VIMNMX3, S - Y runs on the FMA pipe
-                    const int wn = __vimax3_s32(wu, W[k], fma_add(sr, one, mY));
-                    const int xn = kill_fma(sr, wn, mOE, one, zero);
+                    // live iff S_raw >= thr = max(W_up, W_left) (reading R3); W = max(thr, S_raw - Y) equals
+                    // max(thr, S_live - Y) because a dead cell has S_raw - Y < S_raw < thr.  thr comes from the
+                    // row above and the previous column (ready before S), so the dependent chain after S is one
+                    // ISETP + the FMA-pipe kill, and W (one VIADDMNMX from S) is off the chain (measured 637 ->
+                    // 621 ms on C2 against W-first with the live test S >= W)
+                    const int thr = imax(wu, W[k]);
+                    const int xn = kill_fma(sr, thr, mOE, one, zero);
+                    const int wn = __viaddmax_s32(sr, mY, thr);
                     if constexpr (MODE == MODE_EXEC) {
                         const uint32_t code = cell_code(h, d, iv, du, xu, I[k], X[k], E);
                         cw |= code << ((((j % SPW) * R) + k) * 4);
