@@ -458,8 +458,10 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
         const char* e = getenv("FASTZ_POOL_MB");
         if (e) {
             budget_words = std::max<long long>(atoll(e), 1) * (1LL << 20) / 4;
+        } else if (words <= (long long)(c->codes.cap / 4)) {
+            budget_words = words;  // the pool already holds one wave: no memory query on the common path
         } else {
-            size_t fr = 0, tot = 0;
+            size_t fr = 0, tot = 0;  // cudaMemGetInfo costs milliseconds: only when the pool must grow
             cudaMemGetInfo(&fr, &tot);
             budget_words = (long long)((fr + c->codes.cap) / 2 / 4);
         }
