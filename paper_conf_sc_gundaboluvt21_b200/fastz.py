@@ -235,6 +235,29 @@ def fastz_int_peak(device: int = 0, ms: float = 200.0):
     return ops.value, mhz.value
 
 
+_ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+_FREE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
+
+
+def torch_allocator_hooks(device: int = 0):
+    """(dev_alloc, dev_free) C callbacks that route the context's device memory through PyTorch's caching
+    allocator (on the context's stream), so freed pools are reused by later contexts without cudaMalloc/cudaFree.
+    Keep the returned objects alive as long as the context."""
+    import torch
+
+    def _alloc(nbytes, stream, user):
+        try:
+            return torch.cuda.caching_allocator_alloc(int(nbytes), device, stream or 0)
+        except Exception:  # out of memory: the library reports FASTZ_ENOMEM
+            return None
+
+    def _free(ptr, stream, user):
+        if ptr:
+            torch.cuda.caching_allocator_delete(ptr)
+
+    return _ALLOC_FN(_alloc), _FREE_FN(_free)
+
+
 # ----------------------------------------------------------------------------------- convenience class
 
 @dataclass
@@ -252,8 +275,13 @@ class Aligner:
     """One context (device + stream + packed sequences).  ``extend`` returns host results; ``extend_only``
     leaves them on the device (for timing / NCCL gathers)."""
 
-    def __init__(self, target, query, params: fastz_params | None = None, device: int = 0, stream=None, **kw):
+    def __init__(self, target, query, params: fastz_params | None = None, device: int = 0, stream=None,
+                 torch_alloc: bool = False, **kw):
         self.params = params if params is not None else fastz_default_params(**kw)
+        if torch_alloc:  # device memory through PyTorch's caching allocator (fastz_params.dev_alloc / dev_free)
+            self._hooks = torch_allocator_hooks(device)
+            self.params.dev_alloc = ctypes.cast(self._hooks[0], ctypes.c_void_p)
+            self.params.dev_free = ctypes.cast(self._hooks[1], ctypes.c_void_p)
         if stream is None:
             try:
                 import torch

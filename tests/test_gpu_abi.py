@@ -102,3 +102,21 @@ def test_results_pinned_equal_results():
         p2 = a.results_pinned()
         assert len(p2.rec) == 10
         assert all(p2.cigar_of(s) == r.cigar_of(s) for s in range(10))
+
+
+def test_torch_caching_allocator_hooks():
+    """fastz_params.dev_alloc / dev_free routed through PyTorch's caching allocator: identical results, and the
+    context's blocks return to PyTorch's cache on destroy (reused by the next context)."""
+    w = _w()
+    with fastz.Aligner(w.T, w.Q) as a:
+        ra = a.extend(w.seeds)
+    before = torch.cuda.memory_allocated()
+    with fastz.Aligner(w.T, w.Q, torch_alloc=True) as b:
+        rb = b.extend(w.seeds)
+        assert torch.cuda.memory_allocated() > before      # the context's buffers live in PyTorch's pool
+        hs, an, _ = b.find_hsps(hspthresh=500)
+    assert np.array_equal(ra.rec, rb.rec) and ra.cigar == rb.cigar
+    assert torch.cuda.memory_allocated() == before         # all returned on destroy
+    with fastz.Aligner(w.T, w.Q, torch_alloc=True) as c:   # reuses the cached blocks
+        rc = c.extend(w.seeds)
+    assert np.array_equal(ra.rec, rc.rec)
