@@ -231,8 +231,11 @@ __device__ __forceinline__ void inspect_body(const DevParams& P, const Batch& b,
     }
 }
 
+#ifndef INSPECT_ATTR
+#define INSPECT_ATTR __launch_bounds__(WARPS * 32)
+#endif
 template <int R>
-__global__ void __launch_bounds__(WARPS * 32) k_inspect(DevParams P, Batch b, int4* ring, int rmask, SideArrays sa,
+__global__ void INSPECT_ATTR k_inspect(DevParams P, Batch b, int4* ring, int rmask, SideArrays sa,
                                                          ExecPlan pl, int budget) {
     inspect_body<R, false>(P, b, ring, rmask, sa, pl, budget);
 }
