@@ -240,7 +240,10 @@ __global__ void INSPECT_ATTR k_inspect(DevParams P, Batch b, int4* ring, int rma
     inspect_body<R, false>(P, b, ring, rmask, sa, pl, budget);
 }
 template <int R>
-__global__ void __maxnreg__(72) k_inspect_n(DevParams P, Batch b, int4* ring, int rmask,
+#ifndef INSPECT_N_MAXREG
+#define INSPECT_N_MAXREG 72
+#endif
+__global__ void __maxnreg__(INSPECT_N_MAXREG) k_inspect_n(DevParams P, Batch b, int4* ring, int rmask,
                                                                            SideArrays sa, ExecPlan pl, int budget) {
     inspect_body<R, true>(P, b, ring, rmask, sa, pl, budget);
 }
