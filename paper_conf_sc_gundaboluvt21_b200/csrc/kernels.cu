@@ -303,8 +303,13 @@ __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int
 // Trimmed executor: the DP over [0,i*]x[0,j*] only, writing traceback codes.  Length binning
 // as a schedule: the CTAs first take the long sides (bins >= 3, block per side, strips pipelined
 // across the CTA's warps), then every warp takes short sides (bins 1-2, warp per side), larger bins first.
+#ifdef EXECUTE_MIN_BLOCKS
+#define EXECUTE_ATTR __launch_bounds__(WARPS * 32, EXECUTE_MIN_BLOCKS)
+#else
+#define EXECUTE_ATTR __launch_bounds__(WARPS * 32)
+#endif
 template <int R, bool NM>
-__global__ void __launch_bounds__(WARPS * 32) k_execute(DevParams P, Batch b, int4* ring, int rmask,
+__global__ void EXECUTE_ATTR k_execute(DevParams P, Batch b, int4* ring, int rmask,
                                                          SideArrays sa, ExecPlan pl, int lo, int hi, int nblock,
                                                          long long base, Outputs out) {
     __shared__ SmemDP sm;
