@@ -256,6 +256,23 @@ def run_fastz(args, ws, rank, local):
     al2 = fastz.Aligner(w.T, w.Q, device=local, stream=stream.cuda_stream, torch_alloc=True)
     al2.extend(np.ascontiguousarray(shard))
     wall_s = time.perf_counter() - t0
+    # NEXT-4 stage on the same pair (rank 0, untimed by the step clock): seeding + ungapped filter
+    seeding = None
+    if rank == 0:
+        try:
+            al2.find_hsps()
+            ts = []
+            for _ in range(3):
+                torch.cuda.synchronize()
+                t1 = time.perf_counter()
+                hs, _an, hits = al2.find_hsps()
+                torch.cuda.synchronize()
+                ts.append(time.perf_counter() - t1)
+            seeding = {"stage": "seeding + ungapped filter (fastz_find_hsps: 12of19 spaced seeds + transitions, "
+                                "x-drop 910, HSP >= 3000), whole pair", "ms": min(ts) * 1e3, "hits": hits,
+                       "hsps": int(len(hs)), "query_mbp_per_s": len(w.Q) / min(ts) / 1e6}
+        except Exception as e:  # reported, never fatal for the headline line
+            seeding = {"error": str(e)[:200]}
     al2.close()
 
     t = torch.tensor([ms, e2e_ms, float(cells), float(n)], dtype=torch.float64, device=dev)
@@ -295,6 +312,7 @@ def run_fastz(args, ws, rank, local):
                 "h2d_bytes_per_step": int(n * 16), "d2h_bytes_per_step": int(d2h)},
         "gpu_launches": launches,
         "genome_pair_wall_s": wall_s,
+        "seeding": seeding,
         "roofline": {"bound": "alu", "kernel": "k_inspect", "achieved": achieved / 1e12, "peak": peak_ops / 1e12,
                      "unit": "Tops/s (INT32 lane ops)", "frac": achieved / peak_ops, "traffic": traffic,
                      "ops_per_cell": OPS_PER_CELL, "inspector_ms": insp_ms,
