@@ -273,6 +273,26 @@ def run_fastz(args, ws, rank, local):
                        "hsps": int(len(hs)), "query_mbp_per_s": len(w.Q) / min(ts) / 1e6}
         except Exception as e:  # reported, never fatal for the headline line
             seeding = {"error": str(e)[:200]}
+    # NEXT-3 post-pass on the same batch (rank 0, untimed by the step clock): redundant-alignment marking
+    dedup = None
+    if rank == 0:
+        try:
+            al2.mark_redundant()
+            ts = []
+            for _ in range(3):
+                ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                torch.cuda.synchronize()
+                ev0.record(stream)
+                _red, nred = al2.mark_redundant()
+                ev1.record(stream)
+                ev1.synchronize()
+                ts.append(ev0.elapsed_time(ev1))
+            nk = int((al2.results().rec["flags"] & fastz.FLAG_ABOVE_K != 0).sum())
+            dedup = {"stage": "redundant-alignment post-pass (fastz_mark_redundant, reading R14), whole batch, "
+                              "incl. the D2H of the per-seed marks", "ms": min(ts), "above_k": nk,
+                     "redundant": int(nred)}
+        except Exception as e:
+            dedup = {"error": str(e)[:200]}
     al2.close()
 
     t = torch.tensor([ms, e2e_ms, float(cells), float(n)], dtype=torch.float64, device=dev)
@@ -313,6 +333,7 @@ def run_fastz(args, ws, rank, local):
         "gpu_launches": launches,
         "genome_pair_wall_s": wall_s,
         "seeding": seeding,
+        "dedup": dedup,
         "roofline": {"bound": "alu", "kernel": "k_inspect", "achieved": achieved / 1e12, "peak": peak_ops / 1e12,
                      "unit": "Tops/s (INT32 lane ops)", "frac": achieved / peak_ops, "traffic": traffic,
                      "ops_per_cell": OPS_PER_CELL, "inspector_ms": insp_ms,

@@ -100,6 +100,7 @@ typedef struct {
 #define FASTZ_FLAG_RIGHT_EAGER 4u /* right side traced back eagerly */
 #define FASTZ_FLAG_OVERFLOW 8u  /* a one-sided peak score reached 2^29 */
 #define FASTZ_FLAG_NO_CIGAR 16u /* CIGAR skipped (FASTZ_OPT_TRACEBACK_ABOVE_K and score < K) */
+#define FASTZ_FLAG_REDUNDANT 32u /* set by fastz_mark_redundant: dominated by another record (reading R14) */
 
 /* One alignment per seed, in seed order (64 bytes). */
 typedef struct {
@@ -222,6 +223,21 @@ void fastz_default_seed_params(fastz_seed_params *sp);
  */
 int fastz_find_hsps(fastz_ctx *c, const fastz_seed_params *sp, fastz_hsp *hsps, fastz_seed *anchors, int64_t cap,
                     int64_t *n_out, int64_t *n_hits);
+
+/*
+ * Redundant-alignment post-pass.  PAPER.md P:110: LASTZ "terminates an ongoing seed
+ * extension upon reaching a previously-discovered alignment"; that skip is sequential-order dependent,
+ * so FastZ extends every seed.  This call applies it after the fact, order-free (reading R14), on the
+ * last batch's device records: among records with FASTZ_FLAG_ABOVE_K, record b dominates record a (a != b) iff
+ * b.t_start <= a.t_start, a.t_end <= b.t_end, b.q_start <= a.q_start, a.q_end <= b.q_end, b.score >= a.score,
+ * and (the boxes differ, or b.score > a.score, or b's seed index is lower).  A dominated record is redundant:
+ * FASTZ_FLAG_REDUNDANT is set in its device record (a later fastz_get_alignments returns it; the bit is
+ * recomputed, not accumulated, on every call) and, if `redundant` (host, may be NULL) is given, redundant[s] =
+ * 1, else 0, for every seed s (cap >= n, else FASTZ_ETRUNC and nothing is written).  *n_redundant (may be
+ * NULL) receives the count.  Records below K are never marked.  Synchronizes the stream.  ESTATE before any
+ * extend call; ENOMEM / ECUDA as elsewhere.
+ */
+int fastz_mark_redundant(fastz_ctx *c, uint8_t *redundant, int64_t cap, int64_t *n_redundant);
 
 /* Release everything; NULL-safe. */
 void fastz_destroy(fastz_ctx *c);

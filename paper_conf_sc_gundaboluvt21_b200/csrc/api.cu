@@ -60,6 +60,8 @@ struct fastz_ctx {
     // seeding (fastz_find_hsps)
     DBuf s_kin, s_kout, s_pin, s_pout, s_start, s_cnt, s_off, s_hits, s_hsp, s_keep, s_sel, s_list, s_list2,
         s_k1, s_k2, s_i1, s_i2, s_flag, s_pos, s_out, s_anch, s_tmp;
+    // redundant-alignment post-pass (fastz_mark_redundant)
+    DBuf r_k1, r_k2, r_i1, r_i2, r_box, r_sc, r_red, r_tmp, r_cnt;
     int R = 4, grid = 0, nslots = 0, rmask = 0;
     int64_t n = 0, cigar_bytes = 0, nexec = 0;
     int nwaves = 0;
@@ -297,7 +299,8 @@ void fastz_destroy(fastz_ctx* c) {
                     &c->stab, &c->runs, &c->nruns, &c->ciglen, &c->cigar, &c->recs, &c->cells, &c->ring,
                     &c->small, &c->s_kin, &c->s_kout, &c->s_pin, &c->s_pout, &c->s_start, &c->s_cnt, &c->s_off,
                     &c->s_hits, &c->s_hsp, &c->s_keep, &c->s_sel, &c->s_list, &c->s_list2, &c->s_k1, &c->s_k2,
-                    &c->s_i1, &c->s_i2, &c->s_flag, &c->s_pos, &c->s_out, &c->s_anch, &c->s_tmp};
+                    &c->s_i1, &c->s_i2, &c->s_flag, &c->s_pos, &c->s_out, &c->s_anch, &c->s_tmp,
+                    &c->r_k1, &c->r_k2, &c->r_i1, &c->r_i2, &c->r_box, &c->r_sc, &c->r_red, &c->r_tmp, &c->r_cnt};
     for (DBuf* b : bufs) dfree(c, *b);
     if (c->ev_ok)
         for (auto& e : c->ev) cudaEventDestroy(e);
@@ -619,6 +622,34 @@ int fastz_get_stats(fastz_ctx* c, fastz_stats* s) {
     S.ms_combine = el(5, 6);
     S.ms_total = el(0, 6);
     *s = S;
+    return 0;
+}
+
+int fastz_mark_redundant(fastz_ctx* c, uint8_t* redundant, int64_t cap, int64_t* n_redundant) {
+    if (!c) return fail(FASTZ_EINVAL, "ctx is NULL");
+    if (!c->have) return fail(FASTZ_ESTATE, "no results: call fastz_extend_seeds first");
+    if (redundant && cap < c->n) return fail(FASTZ_ETRUNC, "cap < n");
+    CK(cudaSetDevice(c->device));
+    const int n = (int)c->n;
+    const size_t m = (size_t)std::max(n, 1);
+    const size_t tb = redundant_tmp_bytes(n);
+    AL(r_k1, m * 4);
+    AL(r_k2, m * 4);
+    AL(r_i1, m * 4);
+    AL(r_i2, m * 4);
+    AL(r_box, m * 16);
+    AL(r_sc, m * 8);
+    AL(r_red, m);
+    AL(r_tmp, tb);
+    AL(r_cnt, 16);
+    CK(launch_redundant(c->recs.p, n, c->r_tmp.p, c->r_tmp.cap, P_<uint32_t>(c->r_k1), P_<uint32_t>(c->r_k2),
+                        P_<int>(c->r_i1), P_<int>(c->r_i2), P_<int4>(c->r_box), P_<int2>(c->r_sc),
+                        P_<unsigned char>(c->r_red), P_<int>(c->r_cnt), c->stream));
+    int cnt[3] = {0, 0, 0};
+    CK(cudaMemcpyAsync(cnt, c->r_cnt.p, sizeof(cnt), cudaMemcpyDeviceToHost, c->stream));
+    if (redundant && n) CK(cudaMemcpyAsync(redundant, c->r_red.p, (size_t)n, cudaMemcpyDeviceToHost, c->stream));
+    CK(cudaStreamSynchronize(c->stream));
+    if (n_redundant) *n_redundant = cnt[2];
     return 0;
 }
 

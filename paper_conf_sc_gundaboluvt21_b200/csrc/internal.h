@@ -73,6 +73,10 @@ cudaError_t launch_bin(int R, const DevParams& P, const SideArrays& sa, int nsid
                        size_t scan_tmp_bytes, long long* tmp_a, long long* tmp_b, long long* tmp_c,
                        cudaStream_t st);
 size_t scan_tmp_bytes(int n);
+// redundant-alignment post-pass (dedup.cu; NEXT-3, reading R14)
+size_t redundant_tmp_bytes(int n);
+cudaError_t launch_redundant(void* recs, int n, void* tmp, size_t tmp_bytes, uint32_t* k1, uint32_t* k2, int* i1,
+                             int* i2, int4* box, int2* sc, unsigned char* red, int* counters, cudaStream_t st);
 cudaError_t launch_execute(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
                            const SideArrays& sa, const ExecPlan& pl, int lo, int hi, int nblock, long long base,
                            const Outputs& o,

@@ -19,13 +19,14 @@ LIB_PATH = os.path.join(HERE, "libfastz.so")
 
 FASTZ_OK, FASTZ_EINVAL, FASTZ_EBASE, FASTZ_ERANGE = 0, -1, -2, -3
 FASTZ_ENOMEM, FASTZ_ECUDA, FASTZ_ETRUNC, FASTZ_ESTATE = -4, -5, -6, -7
-FLAG_ABOVE_K, FLAG_LEFT_EAGER, FLAG_RIGHT_EAGER, FLAG_OVERFLOW, FLAG_NO_CIGAR = 1, 2, 4, 8, 16
+FLAG_ABOVE_K, FLAG_LEFT_EAGER, FLAG_RIGHT_EAGER, FLAG_OVERFLOW, FLAG_NO_CIGAR, FLAG_REDUNDANT = 1, 2, 4, 8, 16, 32
 OPT_NO_EAGER, OPT_NO_TRIM, OPT_NO_BINNING, OPT_NO_BLOCK, OPT_TRACEBACK_ABOVE_K = 1, 2, 4, 8, 16
 
 # names declared in include/fastz.h (checked by tests/test_abi.py against the header)
 EXPORTS = ["fastz_default_params", "fastz_create", "fastz_extend_seeds", "fastz_get_alignments",
            "fastz_get_alignments_device", "fastz_get_sides", "fastz_census", "fastz_get_stats",
-           "fastz_destroy", "fastz_strerror", "fastz_int_peak", "fastz_default_seed_params", "fastz_find_hsps"]
+           "fastz_destroy", "fastz_strerror", "fastz_int_peak", "fastz_default_seed_params", "fastz_find_hsps",
+           "fastz_mark_redundant"]
 
 
 class FastzError(RuntimeError):
@@ -87,6 +88,7 @@ def lib() -> ctypes.CDLL:
                                               ctypes.POINTER(i64)]
     L.fastz_get_sides.argtypes = [vp, vp, vp, vp, vp, i64]
     L.fastz_census.argtypes = [vp, vp, i64]
+    L.fastz_mark_redundant.argtypes = [vp, vp, i64, ctypes.POINTER(i64)]
     L.fastz_get_stats.argtypes = [vp, ctypes.POINTER(fastz_stats)]
     L.fastz_destroy.argtypes = [vp]
     L.fastz_destroy.restype = None
@@ -190,6 +192,14 @@ def fastz_census(ctx: int, n: int) -> np.ndarray:
     cells = np.zeros(max(2 * n, 1), np.int64)
     _check(lib().fastz_census(ctx, cells.ctypes.data, 2 * n))
     return cells[:2 * n]
+
+
+def fastz_mark_redundant(ctx: int, n: int):
+    """Redundant-alignment post-pass (NEXT-3, reading R14) on the last batch: returns (uint8[n] marks, count)."""
+    red = np.zeros(max(n, 1), np.uint8)
+    cnt = ctypes.c_int64()
+    _check(lib().fastz_mark_redundant(ctx, red.ctypes.data, n, ctypes.byref(cnt)))
+    return red[:n], cnt.value
 
 
 def fastz_get_stats(ctx: int) -> dict:
@@ -330,6 +340,10 @@ class Aligner:
     def find_hsps(self, **seed_params):
         """Seeding + ungapped filter on this context's sequences (NEXT-4): (hsps, anchors, hits)."""
         return fastz_find_hsps(self.ctx, fastz_default_seed_params(**seed_params))
+
+    def mark_redundant(self):
+        """fastz_mark_redundant on the last batch: (uint8[n] marks, count); sets FLAG_REDUNDANT in the records."""
+        return fastz_mark_redundant(self.ctx, self.n)
 
     def census(self) -> np.ndarray:
         return fastz_census(self.ctx, self.n)
