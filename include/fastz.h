@@ -239,6 +239,20 @@ int fastz_find_hsps(fastz_ctx *c, const fastz_seed_params *sp, fastz_hsp *hsps, 
  */
 int fastz_mark_redundant(fastz_ctx *c, uint8_t *redundant, int64_t cap, int64_t *n_redundant);
 
+/*
+ * The same post-pass (reading R14) on any caller-owned record set, without a context -- e.g. the records of
+ * several batches or ranks gathered in one array (paper_conf_sc_gundaboluvt21_b200/dist.py).  recs[n] holds
+ * fastz_alignment records (host memory if recs_on_device == 0, else device memory of `device`); only score,
+ * flags, t_start/t_end and q_start/q_end are read, and FASTZ_FLAG_REDUNDANT is recomputed in place in every
+ * record's flags.  The seed index of the tie rule is the record's position in the array; coordinates must lie
+ * in [0, 2^31) as fastz_extend_seeds produces them.  redundant (host,
+ * may be NULL) receives n marks, *n_redundant (may be NULL) the count.  Uses a private stream and scratch
+ * device memory (cudaMalloc), freed before returning; synchronous.  EINVAL (n < 0, n >= 2^31, recs NULL with
+ * n > 0), ENOMEM, ECUDA.
+ */
+int fastz_mark_redundant_records(fastz_alignment *recs, int64_t n, int recs_on_device, uint8_t *redundant,
+                                 int64_t *n_redundant, int device);
+
 /* Release everything; NULL-safe. */
 void fastz_destroy(fastz_ctx *c);
 

@@ -653,6 +653,48 @@ int fastz_mark_redundant(fastz_ctx* c, uint8_t* redundant, int64_t cap, int64_t*
     return 0;
 }
 
+int fastz_mark_redundant_records(fastz_alignment* recs, int64_t n, int recs_on_device, uint8_t* redundant,
+                                 int64_t* n_redundant, int device) {
+    if (n < 0 || n > INT_MAX) return fail(FASTZ_EINVAL, "n must be in [0, 2^31)");
+    if (n && !recs) return fail(FASTZ_EINVAL, "recs is NULL");
+    if (n_redundant) *n_redundant = 0;
+    if (n == 0) return 0;
+    CK(cudaSetDevice(device));
+    struct Scratch {  // released on every return path
+        void* p = nullptr;
+        cudaStream_t s = nullptr;
+        ~Scratch() {
+            if (s) cudaStreamSynchronize(s);
+            if (p) cudaFree(p);
+            if (s) cudaStreamDestroy(s);
+        }
+    } sc;
+    CK(cudaStreamCreateWithFlags(&sc.s, cudaStreamNonBlocking));
+    const size_t m = (size_t)n;
+    auto up = [](size_t b) { return (b + 255) & ~(size_t)255; };
+    const size_t tb = redundant_tmp_bytes((int)n);
+    const size_t o_rec = 0, o_k1 = o_rec + (recs_on_device ? 0 : up(m * sizeof(fastz_alignment)));
+    const size_t o_k2 = o_k1 + up(m * 4), o_i1 = o_k2 + up(m * 4), o_i2 = o_i1 + up(m * 4);
+    const size_t o_box = o_i2 + up(m * 4), o_sc = o_box + up(m * 16), o_red = o_sc + up(m * 8);
+    const size_t o_cnt = o_red + up(m), o_tmp = o_cnt + 256, total = o_tmp + up(tb);
+    CK(cudaMalloc(&sc.p, total));
+    char* base = static_cast<char*>(sc.p);
+    void* drecs = recs_on_device ? (void*)recs : (void*)(base + o_rec);
+    if (!recs_on_device)
+        CK(cudaMemcpyAsync(drecs, recs, m * sizeof(fastz_alignment), cudaMemcpyHostToDevice, sc.s));
+    CK(launch_redundant(drecs, (int)n, base + o_tmp, up(tb), (uint32_t*)(base + o_k1), (uint32_t*)(base + o_k2),
+                        (int*)(base + o_i1), (int*)(base + o_i2), (int4*)(base + o_box), (int2*)(base + o_sc),
+                        (unsigned char*)(base + o_red), (int*)(base + o_cnt), sc.s));
+    int cnt[3] = {0, 0, 0};
+    CK(cudaMemcpyAsync(cnt, base + o_cnt, sizeof(cnt), cudaMemcpyDeviceToHost, sc.s));
+    if (redundant) CK(cudaMemcpyAsync(redundant, base + o_red, m, cudaMemcpyDeviceToHost, sc.s));
+    if (!recs_on_device)
+        CK(cudaMemcpyAsync(recs, drecs, m * sizeof(fastz_alignment), cudaMemcpyDeviceToHost, sc.s));
+    CK(cudaStreamSynchronize(sc.s));
+    if (n_redundant) *n_redundant = cnt[2];
+    return 0;
+}
+
 int fastz_int_peak(int device, float ms, double* ops_per_s, double* sm_clock_mhz) {
     if (!ops_per_s || !sm_clock_mhz) return fail(FASTZ_EINVAL, "NULL argument");
     CK(int_peak_run(device, ms, ops_per_s, sm_clock_mhz));

@@ -116,9 +116,12 @@ def cuda_extend_fn(device: int):
 
 
 def extend_genome_pair(T: bytes | None, Q: bytes | None, seeds: np.ndarray | None, params=None, group=None,
-                       extend_fn=None, src: int = 0):
+                       extend_fn=None, src: int = 0, mark_redundant: bool = False, mark_fn=None):
     """Collective: every rank calls it; only ``src`` needs real inputs.  Returns (records, cigar) on ``src``
-    (seed order), (None, None) elsewhere."""
+    (seed order), (None, None) elsewhere.  ``mark_redundant``: after the gather, ``src`` runs the
+    redundant-alignment post-pass (NEXT-3, reading R14) over the WHOLE record set -- the marks depend on every
+    record, so they cannot be taken per shard -- setting FLAG_REDUNDANT in place (``mark_fn(rec)``, default the
+    CUDA ``fastz_mark_redundant_records`` on the current device)."""
     rank, world = dist.get_rank(group), dist.get_world_size(group)
     T = broadcast_bytes(T, src, group)
     Q = broadcast_bytes(Q, src, group)
@@ -129,4 +132,11 @@ def extend_genome_pair(T: bytes | None, Q: bytes | None, seeds: np.ndarray | Non
     if extend_fn is None:
         extend_fn = cuda_extend_fn(torch.cuda.current_device())
     rec, cig = extend_fn(T, Q, seeds[idx], params)
-    return gather_results(idx, rec, cig, n, group, src)
+    out_rec, out_cig = gather_results(idx, rec, cig, n, group, src)
+    if mark_redundant and out_rec is not None:
+        out_rec = np.ascontiguousarray(out_rec)
+        if mark_fn is None:
+            fastz.fastz_mark_redundant_records(out_rec, torch.cuda.current_device())
+        else:
+            mark_fn(out_rec)
+    return out_rec, out_cig

@@ -26,7 +26,7 @@ OPT_NO_EAGER, OPT_NO_TRIM, OPT_NO_BINNING, OPT_NO_BLOCK, OPT_TRACEBACK_ABOVE_K =
 EXPORTS = ["fastz_default_params", "fastz_create", "fastz_extend_seeds", "fastz_get_alignments",
            "fastz_get_alignments_device", "fastz_get_sides", "fastz_census", "fastz_get_stats",
            "fastz_destroy", "fastz_strerror", "fastz_int_peak", "fastz_default_seed_params", "fastz_find_hsps",
-           "fastz_mark_redundant"]
+           "fastz_mark_redundant", "fastz_mark_redundant_records"]
 
 
 class FastzError(RuntimeError):
@@ -89,6 +89,7 @@ def lib() -> ctypes.CDLL:
     L.fastz_get_sides.argtypes = [vp, vp, vp, vp, vp, i64]
     L.fastz_census.argtypes = [vp, vp, i64]
     L.fastz_mark_redundant.argtypes = [vp, vp, i64, ctypes.POINTER(i64)]
+    L.fastz_mark_redundant_records.argtypes = [vp, i64, i32, vp, ctypes.POINTER(i64), i32]
     L.fastz_get_stats.argtypes = [vp, ctypes.POINTER(fastz_stats)]
     L.fastz_destroy.argtypes = [vp]
     L.fastz_destroy.restype = None
@@ -199,6 +200,19 @@ def fastz_mark_redundant(ctx: int, n: int):
     red = np.zeros(max(n, 1), np.uint8)
     cnt = ctypes.c_int64()
     _check(lib().fastz_mark_redundant(ctx, red.ctypes.data, n, ctypes.byref(cnt)))
+    return red[:n], cnt.value
+
+
+def fastz_mark_redundant_records(rec: np.ndarray, device: int = 0):
+    """Context-free post-pass (reading R14) on a host ALIGN_DTYPE array: sets FLAG_REDUNDANT in rec["flags"] in
+    place (the array must be C-contiguous) and returns (uint8[n] marks, count)."""
+    if rec.dtype != ALIGN_DTYPE or not rec.flags["C_CONTIGUOUS"] or not rec.flags["WRITEABLE"]:
+        raise ValueError("rec must be a writeable C-contiguous ALIGN_DTYPE array")
+    n = len(rec)
+    red = np.zeros(max(n, 1), np.uint8)
+    cnt = ctypes.c_int64()
+    _check(lib().fastz_mark_redundant_records(rec.ctypes.data if n else None, n, 0, red.ctypes.data,
+                                              ctypes.byref(cnt), device))
     return red[:n], cnt.value
 
 

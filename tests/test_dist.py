@@ -31,6 +31,11 @@ def _oracle_fn(T, Q, seeds, params):
     return out, r.cigar
 
 
+def _oracle_mark(rec):
+    from oracle import dedup
+    rec["flags"] |= dedup.redundant(rec).astype(np.uint32) << 5   # FLAG_REDUNDANT = 32
+
+
 def _worker(rank, world, port, q):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
@@ -39,7 +44,8 @@ def _worker(rank, world, port, q):
         from synth import genome
         w = genome.small_pair(21, length=8000, n_seeds=90)
         rec, cig = fzdist.extend_genome_pair(w.T if rank == 0 else None, w.Q if rank == 0 else None,
-                                             w.seeds if rank == 0 else None, extend_fn=_oracle_fn)
+                                             w.seeds if rank == 0 else None, extend_fn=_oracle_fn,
+                                             mark_redundant=True, mark_fn=_oracle_mark)
         if rank == 0:
             q.put((rec.tobytes(), cig))
     finally:
@@ -70,4 +76,7 @@ def test_gloo_world2_matches_single_process(world):
         assert p.exitcode == 0
     w = genome.small_pair(21, length=8000, n_seeds=90)
     ref_rec, ref_cig = _oracle_fn(w.T, w.Q, w.seeds, None)
+    # the post-pass runs once over the gathered WHOLE set (marks depend on every record, not one shard's)
+    _oracle_mark(ref_rec)
+    assert (ref_rec["flags"] & 32).any()
     assert rec_bytes == ref_rec.tobytes() and cig == ref_cig

@@ -100,3 +100,32 @@ def test_c2_full_batch_maximality():
         rec = al.results().rec
     assert cnt == int(red.sum()) and cnt > 0
     assert np.array_equal(red, maximal_marks(rec))
+
+
+def oracle_records(o):
+    rec = np.zeros(len(o.rec), dtype=fastz.ALIGN_DTYPE)
+    for f in ("score", "left_score", "right_score", "flags", "t_start", "t_end", "q_start", "q_end"):
+        rec[f] = o.rec[f]
+    return rec
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_context_free_records_match_oracle(seed):
+    """fastz_mark_redundant_records on ORACLE records held on the host (gathered-set use, dist.py)."""
+    w = genome.small_pair(40 + seed, length=20_000, n_seeds=300)
+    o = core.extend(w.T, w.Q, w.seeds, oparams(gapped_threshold=1000))
+    rec = oracle_records(o)
+    rec["flags"] |= fastz.FLAG_REDUNDANT * (np.arange(len(rec)) % 2).astype(np.uint32)  # stale bits are recomputed
+    red, cnt = fastz.fastz_mark_redundant_records(rec)
+    exp = dedup.redundant(o.rec)
+    assert np.array_equal(red, exp) and cnt == int(exp.sum()) and cnt > 0
+    assert np.array_equal((rec["flags"] & fastz.FLAG_REDUNDANT) != 0, exp.astype(bool))
+    assert np.array_equal(rec["flags"] & ~np.uint32(fastz.FLAG_REDUNDANT), o.rec["flags"].astype(np.uint32))
+
+
+def test_context_free_empty_and_bad_args():
+    rec = np.zeros(0, dtype=fastz.ALIGN_DTYPE)
+    red, cnt = fastz.fastz_mark_redundant_records(rec)
+    assert len(red) == 0 and cnt == 0
+    with pytest.raises(ValueError):
+        fastz.fastz_mark_redundant_records(np.zeros(3, np.int64))

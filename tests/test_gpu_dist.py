@@ -25,10 +25,12 @@ def test_nccl_world1_matches_oracle():
                             device_id=torch.device("cuda", 0))
     try:
         w = genome.small_pair(31, length=20000, n_seeds=150)
-        rec, cig = fzdist.extend_genome_pair(w.T, w.Q, w.seeds)
+        rec, cig = fzdist.extend_genome_pair(w.T, w.Q, w.seeds, mark_redundant=True)
     finally:
         dist.destroy_process_group()
     o = core.extend(w.T, w.Q, w.seeds, oparams())
     for f in ("score", "t_start", "t_end", "q_start", "q_end", "cigar_len"):
         assert np.array_equal(rec[f].astype(np.int64), o.rec[f]), f
     assert cig == o.cigar
+    from oracle import dedup
+    assert np.array_equal((rec["flags"] >> 5) & 1, dedup.redundant(o.rec))

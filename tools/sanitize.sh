@@ -1,5 +1,6 @@
 # compute-sanitizer on a small mixed workload (memcheck, racecheck, synccheck, initcheck); block-per-side forced
-# (so the warp-per-side traceback runs too), plus the seeding stage on both strands
+# (so the warp-per-side traceback runs too), plus the seeding stage on both strands and the redundant-alignment
+# post-pass (K = 0, so every record is a candidate)
 mkdir -p gpurun_out
 python -m paper_conf_sc_gundaboluvt21_b200.build > /dev/null
 cat > /tmp/san_case.py <<'PY'
@@ -13,9 +14,13 @@ with fastz.Aligner(w.T, w.Q) as a:
     a.census()
     hs, an, hits = a.find_hsps(hspthresh=500)
     a.extend(an)
+with fastz.Aligner(w.T, w.Q, fastz.fastz_default_params(gapped_threshold=0)) as d:
+    d.extend(w.seeds)
+    red, nred = d.mark_redundant()
+    d.mark_redundant()
 with fastz.Aligner(w.T, w.Q, fastz.fastz_default_params(options=32)) as b:
     hs2, an2, _ = b.find_hsps(pattern="1101011", hspthresh=300)
-print("ok", len(r.rec), len(hs), len(hs2))
+print("ok", len(r.rec), len(hs), len(hs2), nred)
 PY
 for tool in memcheck racecheck synccheck initcheck; do
   FASTZ_ESCALATE_STRIPS=2 FASTZ_BLOCK_BIN=1 timeout 900 compute-sanitizer --tool $tool --error-exitcode 9 python /tmp/san_case.py > gpurun_out/san_$tool.log 2>&1; echo "$tool rc=$?"; tail -2 gpurun_out/san_$tool.log
