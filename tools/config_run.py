@@ -12,6 +12,9 @@ al = fastz.Aligner(w.T, w.Q)
 al.extend_only(w.seeds)  # warm
 t0 = time.time(); res = al.extend(w.seeds); te = time.time() - t0
 st = al.stats()
+al.mark_redundant()  # NEXT-3 post-pass (reading R14): warm, then timed
+t0 = time.time(); red, nred = al.mark_redundant(); tr = time.time() - t0
+nk = int(((res.rec["flags"] & fastz.FLAG_ABOVE_K) != 0).sum())
 cells = int(al.census().sum())
 rng = np.random.default_rng(cfg)
 idx = np.sort(rng.choice(w.n, min(nsample, w.n), replace=False))
@@ -23,4 +26,5 @@ print(json.dumps({"config": w.name, "seeds": w.n, "tlen": len(w.T), "gen_s": rou
                   "stages_ms": {k: round(st[k], 2) for k in ("ms_total", "ms_inspect", "ms_bin", "ms_execute", "ms_traceback", "ms_combine")},
                   "cells": cells, "GCUPS_e2e": cells / te / 1e9, "GCUPS_device": cells / (st["ms_total"] / 1e3) / 1e9,
                   "bins": st["bin_counts"][:7], "exec_words": st["exec_words"], "sample": len(idx), "parity": bool(ok),
+                  "dedup": {"above_k": nk, "redundant": int(nred), "ms_host": round(tr * 1e3, 2)},
                   "oracle_s": round(to, 1), "oracle_GCUPS": ocells / to / 1e9}))
