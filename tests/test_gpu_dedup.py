@@ -129,3 +129,22 @@ def test_context_free_empty_and_bad_args():
     assert len(red) == 0 and cnt == 0
     with pytest.raises(ValueError):
         fastz.fastz_mark_redundant_records(np.zeros(3, np.int64))
+
+
+def test_context_free_device_records():
+    """recs_on_device = 1: records in device memory (a torch buffer), flags recomputed in place on the GPU."""
+    import ctypes
+
+    import torch
+    w = genome.small_pair(50, length=20_000, n_seeds=300)
+    o = core.extend(w.T, w.Q, w.seeds, oparams(gapped_threshold=0))
+    rec = oracle_records(o)
+    buf = torch.from_numpy(rec.view(np.uint8).copy()).cuda()
+    red = np.zeros(len(rec), np.uint8)
+    cnt = ctypes.c_int64()
+    st = fastz.lib().fastz_mark_redundant_records(buf.data_ptr(), len(rec), 1, red.ctypes.data, ctypes.byref(cnt), 0)
+    assert st == 0
+    exp = dedup.redundant(o.rec)
+    assert np.array_equal(red, exp) and cnt.value == int(exp.sum()) > 0
+    back = buf.cpu().numpy().view(fastz.ALIGN_DTYPE)
+    assert np.array_equal((back["flags"] & fastz.FLAG_REDUNDANT) != 0, exp.astype(bool))
