@@ -60,19 +60,19 @@ __global__ void k_rd_mark(fastz_alignment* __restrict__ recs, int n, const uint3
         if ((long long)keys[mid] < lo_key) lo = mid + 1;
         else hi = mid;
     }
-    bool dom = false;
-    for (int q = lo; q < m && keys[q] <= (uint32_t)a.x; ++q) {
-        if (q == p) continue;
+    auto dominated_by = [&](int q) {
         const int4 b = box[q];
-        if (b.x > a.x || a.y > b.y || b.z > a.z || a.w > b.w) continue;  // box(b) must contain box(a)
+        if (b.x > a.x || a.y > b.y || b.z > a.z || a.w > b.w) return false;  // box(b) must contain box(a)
         const int2 bs = sc[q];
-        if (bs.x < as.x) continue;
+        if (bs.x < as.x) return false;
         const bool same_box = b.x == a.x && b.y == a.y && b.z == a.z && b.w == a.w;
-        if (!same_box || bs.x > as.x || bs.y < as.y) {
-            dom = true;
-            break;
-        }
-    }
+        return !same_box || bs.x > as.x || bs.y < as.y;
+    };
+    // nearest starts first: copies of one alignment (many seeds on one homologous block) share t_start and sit
+    // in seed order just before p, so a redundant copy usually stops at q = p - 1 (C5: 2.98 ms with a forward scan)
+    bool dom = false;
+    for (int q = p - 1; q >= lo && !dom; --q) dom = dominated_by(q);
+    for (int q = p + 1; !dom && q < m && keys[q] <= (uint32_t)a.x; ++q) dom = dominated_by(q);
     if (dom) {
         red[as.y] = 1;
         recs[as.y].flags |= FASTZ_FLAG_REDUNDANT;
