@@ -120,7 +120,9 @@ void fastz_default_params(fastz_params *p);
 
 /*
  * Create a context on `device` using `cuda_stream` (a cudaStream_t; NULL -> the library creates its own
- * non-blocking stream).  `target`/`query` are ASCII (ACGTNacgtn) of tlen/qlen bytes, host or device memory
+ * blocking stream, ordered after work on the legacy default stream).  Device inputs (sequences, seeds) must
+ * be complete with respect to the context's stream when passed: a caller producing them on another stream
+ * synchronizes it (or makes the context's stream wait on it) first.  `target`/`query` are ASCII (ACGTNacgtn) of tlen/qlen bytes, host or device memory
  * (detected with cudaPointerGetAttributes); they are copied, validated and packed to 2 bits per base
  * (forward and reversed copies) plus a 1-bit N mask on the device.  Errors: EINVAL (NULL pointers, bad params), ERANGE (a length
  * < 0 or >= 2^31), EBASE (invalid character), ENOMEM, ECUDA.  On error *out is NULL.
@@ -132,7 +134,8 @@ int fastz_create(const fastz_params *p, const char *target, int64_t tlen, const 
  * Extend n seeds (host or device memory as `seeds_on_device` says; n may be 0).  Runs inspector, binning,
  * executor, traceback and CIGAR assembly on the context's stream; results stay on the device until
  * fastz_get_alignments.  Replaces the results of any previous call.  Errors: EINVAL, ERANGE (a seed out of
- * range -- index in fastz_strerror -- or an explored band wider than the per-warp scratch), ENOMEM, ECUDA.
+ * range -- index in fastz_strerror; the kernels treat such a seed as an empty extension and never read
+ * outside the sequences, and the batch has no results), ENOMEM, ECUDA.
  */
 int fastz_extend_seeds(fastz_ctx *c, const fastz_seed *seeds, int64_t n, int seeds_on_device);
 
@@ -147,7 +150,9 @@ int fastz_get_alignments(fastz_ctx *c, fastz_alignment *out, int64_t out_cap, ch
 
 /*
  * Device-resident view of the last batch (valid until the next extend/destroy): records and CIGAR text in
- * the context's device memory, for callers that keep results on the GPU (e.g. a NCCL gather).
+ * the context's device memory, for callers that keep results on the GPU (e.g. a NCCL gather).  The final
+ * record/CIGAR writes are still queued on the context's stream when fastz_extend_seeds returns: a consumer on
+ * another stream must synchronize the context's stream (or wait on an event recorded on it) before reading.
  */
 int fastz_get_alignments_device(fastz_ctx *c, const fastz_alignment **recs, const char **cigar, int64_t *n,
                                 int64_t *cigar_bytes);
@@ -178,6 +183,11 @@ typedef struct {
     int64_t n_launches;           /* kernels of this library launched by the call (CUB scans excluded) */
     int64_t n_waves;              /* executor/traceback waves under the traceback-pool budget */
     int64_t n_escalated;          /* sides handed from the warp inspector to the block inspector */
+    int64_t n_wide_sides;         /* sides whose explored band outgrew the regular boundary ring and ran with the
+                                     wide ring (very large Y or indel-rich long alignments) */
+    int64_t exec_reserved_words;  /* traceback-pool words reserved for the executor (>= exec_words) */
+    int64_t n_selfcheck_fail;     /* executor self-check failures: S(i*,j*) != inspector score, or code words
+                                     outside a side's reservation (always 0; nonzero -> FASTZ_ECUDA) */
 } fastz_stats;
 int fastz_get_stats(fastz_ctx *c, fastz_stats *s);
 

@@ -56,13 +56,16 @@ struct fastz_ctx {
     bool t_has_n = false, q_has_n = false;
     DBuf seeds, score, ti, qj, flags, eops, bound, maxsw, esc, nstrip;
     DBuf woff, soff, roff, bin, list, counters, totals, tmpa, tmpb, tmpc, scan_tmp, wl, wlo;
-    DBuf codes, stab, runs, nruns, ciglen, cigar, recs, cells, ring, small;
+    DBuf codes, stab, runs, nruns, ciglen, cigar, recs, cells, ring, small, wide, ring2;
     // seeding (fastz_find_hsps)
     DBuf s_kin, s_kout, s_pin, s_pout, s_start, s_cnt, s_off, s_hits, s_hsp, s_keep, s_sel, s_list, s_list2,
         s_k1, s_k2, s_i1, s_i2, s_flag, s_pos, s_out, s_anch, s_tmp;
     // redundant-alignment post-pass (fastz_mark_redundant)
     DBuf r_k1, r_k2, r_i1, r_i2, r_box, r_sc, r_red, r_tmp, r_cnt;
     int R = 4, grid = 0, nslots = 0, rmask = 0;
+    // wide ring of the last batch (sides whose explored band overflowed `ring`): grid2 CTAs x WARPS slots of
+    // rmask2 + 1 entries; nwide sides listed in `wide`
+    int grid2 = 0, rmask2 = 0, nwide = 0;
     int64_t n = 0, cigar_bytes = 0, nexec = 0;
     int nwaves = 0;
     bool have = false;
@@ -223,6 +226,7 @@ ExecPlan make_plan(fastz_ctx* c) {
     p.esc = P_<int>(c->esc);
     p.wl = P_<long long>(c->wl);
     p.wlo = P_<long long>(c->wlo);
+    p.wide = P_<int>(c->wide);
     return p;
 }
 
@@ -297,6 +301,7 @@ void fastz_destroy(fastz_ctx* c) {
                     &c->flags, &c->eops, &c->bound, &c->maxsw, &c->esc, &c->nstrip, &c->woff, &c->soff, &c->roff, &c->bin, &c->list,
                     &c->counters, &c->totals, &c->tmpa, &c->tmpb, &c->tmpc, &c->scan_tmp, &c->wl, &c->wlo, &c->codes,
                     &c->stab, &c->runs, &c->nruns, &c->ciglen, &c->cigar, &c->recs, &c->cells, &c->ring,
+                    &c->wide, &c->ring2,
                     &c->small, &c->s_kin, &c->s_kout, &c->s_pin, &c->s_pout, &c->s_start, &c->s_cnt, &c->s_off,
                     &c->s_hits, &c->s_hsp, &c->s_keep, &c->s_sel, &c->s_list, &c->s_list2, &c->s_k1, &c->s_k2,
                     &c->s_i1, &c->s_i2, &c->s_flag, &c->s_pos, &c->s_out, &c->s_anch, &c->s_tmp,
@@ -324,7 +329,9 @@ int fastz_create(const fastz_params* p, const char* target, int64_t tlen, const 
     if (cuda_stream) {
         c->stream = (cudaStream_t)cuda_stream;
     } else {
-        cudaError_t e = cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking);
+        // a blocking stream: it is ordered after work on the legacy default stream (PyTorch's default), so
+        // device inputs written there (seeds, sequences) are complete before the library reads them
+        cudaError_t e = cudaStreamCreateWithFlags(&c->stream, cudaStreamDefault);
         if (e != cudaSuccess) {
             delete c;
             return fail(FASTZ_ECUDA, std::string("cudaStreamCreate: ") + cudaGetErrorString(e));
@@ -370,6 +377,8 @@ int fastz_create(const fastz_params* p, const char* target, int64_t tlen, const 
     // per-warp boundary ring: the widest explored band is bounded by the query side length; capped
     int64_t want = std::max<int64_t>(std::max<int64_t>(tlen, qlen) + 64, 1024);
     c->rmask = next_pow2(std::min<int64_t>(want, 1 << 15)) - 1;
+    if (const char* e = getenv("FASTZ_RING_ENTRIES"))  // tests: a small ring exercises the wide-band path
+        c->rmask = next_pow2(std::max<int64_t>(atoll(e), 64)) - 1;
     for (auto& e : c->ev) cudaEventCreate(&e);
     c->ev_ok = true;
     *out = c;
@@ -408,6 +417,7 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     AL(wl, std::max<int64_t>(ns, 1) * 8);
     AL(wlo, std::max<int64_t>(ns, 1) * 8);
     AL(nruns, std::max<int64_t>(ns, 1) * 4);
+    AL(wide, std::max<int64_t>(ns, 1) * 4);
     AL(ciglen, std::max<int64_t>(2 * n, 1) * 8);
     AL(recs, std::max<int64_t>(n, 1) * sizeof(fastz_alignment));
     AL(counters, 64 * 4);
@@ -430,7 +440,9 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     SideArrays sa = make_sides(c);
     ExecPlan pl = make_plan(c);
     const int esc = (c->dp.options & OPT_NO_BLOCK) ? 0 : escalate_strips();
-    CK(launch_inspect(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, esc > 0 ? esc : INT_MAX, st));
+    c->nwide = 0;
+    CK(launch_inspect(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, esc > 0 ? esc : INT_MAX,
+                      nullptr, 0, st));
     if (esc > 0) CK(launch_inspect_block(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, st));
     CK(cudaEventRecord(c->ev[2], st));
     CK(launch_bin(c->R, c->dp, sa, (int)ns, pl, c->scan_tmp.p, stb, P_<long long>(c->tmpa), P_<long long>(c->tmpb),
@@ -440,15 +452,62 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     // host sync 1: sizes of the executor's traceback pool
     struct {
         long long totals[5];
-        int counters[24];
+        int counters[26];
         long long bad;
     } h;
-    CK(cudaMemcpyAsync(h.totals, c->totals.p, sizeof(h.totals), cudaMemcpyDeviceToHost, st));
-    CK(cudaMemcpyAsync(h.counters, c->counters.p, sizeof(h.counters), cudaMemcpyDeviceToHost, st));
-    CK(cudaMemcpyAsync(&h.bad, c->small.p, sizeof(h.bad), cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
+    auto sync1 = [&]() -> int {
+        CK(cudaMemcpyAsync(h.totals, c->totals.p, sizeof(h.totals), cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(h.counters, c->counters.p, sizeof(h.counters), cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(&h.bad, c->small.p, sizeof(h.bad), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        return 0;
+    };
+    if ((r = sync1())) return r;
     if (h.bad != LLONG_MAX) return fail(FASTZ_ERANGE, "seed " + std::to_string(h.bad) + " lies outside the sequences");
-    if (h.counters[20]) return fail(FASTZ_ERANGE, "an explored band is wider than the per-warp boundary ring");
+    // Sides whose explored band outgrew the per-warp boundary ring (possible only for very large Y or long
+    // indel-rich alignments; the y-drop rule itself has no width limit) are re-inspected with a ring 4x
+    // wider, repeatedly, up to the query length (a band never spans more than N + 1 columns); the executor then
+    // runs those sides with the same ring.  Memory bounds the number of warp slots of the wide run.
+    int64_t extra_launches = 0;
+    if (h.counters[20]) {
+        int64_t entries = (int64_t)c->rmask + 1;
+        const int64_t cap = next_pow2((int64_t)c->qlen + 64);
+        for (;;) {
+            if (entries >= cap) return fail(FASTZ_ERANGE, "an explored band is wider than the query (internal)");
+            entries = std::min<int64_t>(entries * 4, cap);
+            const int nw = h.counters[24];
+            const size_t slot_bytes = (size_t)entries * sizeof(int4);
+            size_t fr = 0, tot = 0;
+            cudaMemGetInfo(&fr, &tot);
+            const size_t budget = (fr + c->ring2.cap) / 4;
+            int64_t slots = (int64_t)(budget / slot_bytes);
+            slots = std::min<int64_t>(slots, std::min<int64_t>((int64_t)c->nslots, (int64_t)WARPS * nw));
+            const int g2 = (int)(slots / WARPS);
+            if (g2 < 1) return fail(FASTZ_ENOMEM, "no memory for a " + std::to_string(slot_bytes) + "-byte wide ring");
+            AL(ring2, (size_t)g2 * WARPS * slot_bytes);
+            c->grid2 = g2;
+            c->rmask2 = (int)(entries - 1);
+            // re-inspect the listed sides (wide list -> tmp copy, since binning rebuilds it)
+            int* wl = P_<int>(c->tmpc);
+            CK(cudaMemcpyAsync(wl, c->wide.p, (size_t)nw * 4, cudaMemcpyDeviceToDevice, st));
+            CK(cudaMemsetAsync(c->counters.p, 0, 64 * 4, st));
+            CK(launch_inspect(c->R, c->grid2, c->dp, b, P_<int4>(c->ring2), c->rmask2, sa, pl, INT_MAX, wl, nw, st));
+            CK(cudaMemsetAsync(c->counters.p, 0, 64 * 4, st));
+            CK(launch_bin(c->R, c->dp, sa, (int)ns, pl, c->scan_tmp.p, stb, P_<long long>(c->tmpa),
+                          P_<long long>(c->tmpb), P_<long long>(c->tmpc), st));
+            if ((r = sync1())) return r;
+            c->nwide = nw;
+            extra_launches += 6;  // inspect + bin_count, bin_offsets, bin_scatter, list_words, list_offsets
+            if (!h.counters[20]) break;
+        }
+        // the final wide list: every side inspected with the wide ring (SF_WIDE), for the census
+        CK(launch_wide_list(sa, (int)ns, P_<int>(c->wide), P_<int>(c->counters) + 25, st));
+        extra_launches += 1;
+        int nwl = 0;
+        CK(cudaMemcpyAsync(&nwl, P_<int>(c->counters) + 25, 4, cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        c->nwide = nwl;
+    }
     const long long words = h.totals[0], strips = h.totals[1], nrun = h.totals[2];
     c->nexec = h.totals[3];
     const long long nblock = h.totals[4];
@@ -505,7 +564,14 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
         if (w) CK(cudaMemsetAsync(P_<int>(c->counters) + 1, 0, 4, st));
         if (w) CK(cudaMemsetAsync(P_<int>(c->counters) + 23, 0, 4, st));
         CK(launch_execute(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, (int)waves[w].first,
-                          (int)waves[w].second, (int)nblock, wbase[w], o, st));
+                          (int)waves[w].second, (int)nblock, wbase[w], o, 0, st));
+        if (c->nwide) {  // the SF_WIDE sides of this wave, with the wide ring
+            CK(cudaMemsetAsync(P_<int>(c->counters) + 1, 0, 4, st));
+            CK(cudaMemsetAsync(P_<int>(c->counters) + 23, 0, 4, st));
+            CK(launch_execute(c->R, c->grid2, c->dp, b, P_<int4>(c->ring2), c->rmask2, sa, pl, (int)waves[w].first,
+                              (int)waves[w].second, (int)nblock, wbase[w], o, 1, st));
+            extra_launches += 1;
+        }
         if (w == 0) CK(cudaEventRecord(c->ev[4], st));
         CK(launch_traceback(c->R, sa, pl, (int)waves[w].first, (int)waves[w].second, (int)nblock, wbase[w], o, st));
     }
@@ -538,7 +604,8 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     // own kernels: validate, inspect, inspect_block (if escalation on), bin_count, bin_offsets, bin_scatter,
     // list_words, list_offsets, execute per wave, traceback (warp and/or thread variant) per wave, combine_len,
     // combine_total, combine_write
-    S.n_launches = (n > 0 ? 1 + 1 + (esc > 0 ? 1 : 0) + 5 + (int64_t)c->nwaves + tb_launches + 3 : 1);
+    S.n_launches = (n > 0 ? 1 + 1 + (esc > 0 ? 1 : 0) + 5 + (int64_t)c->nwaves + tb_launches + 3 + extra_launches : 1);
+    S.n_wide_sides = c->nwide;
     c->have = true;
     return 0;
 }
@@ -596,7 +663,12 @@ int fastz_census(fastz_ctx* c, int64_t* cells, int64_t cap) {
     CK(cudaMemsetAsync(c->counters.p, 0, 4, c->stream));
     Batch b = make_batch(c);
     CK(launch_census(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, P_<long long>(c->cells),
-                     P_<int>(c->counters), c->stream));
+                     P_<int>(c->counters), nullptr, 0, c->stream));
+    if (c->nwide) {  // sides with a band wider than the regular ring: recount with the wide ring
+        CK(cudaMemsetAsync(c->counters.p, 0, 4, c->stream));
+        CK(launch_census(c->R, c->grid2, c->dp, b, P_<int4>(c->ring2), c->rmask2, P_<long long>(c->cells),
+                         P_<int>(c->counters), P_<int>(c->wide), c->nwide, c->stream));
+    }
     if (c->n) CK(cudaMemcpyAsync(cells, c->cells.p, (size_t)(2 * c->n) * 8, cudaMemcpyDeviceToHost, c->stream));
     CK(cudaStreamSynchronize(c->stream));
     for (int64_t k = 0; k < 2 * c->n; ++k)

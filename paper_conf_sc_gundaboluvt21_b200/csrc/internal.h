@@ -38,11 +38,12 @@ struct ExecPlan {
                          // occupy list[0, totals[4])
     int* counters;       // [0] inspector queue, [1] executor warp queue, [2..8] bin counts, [10..16] bin cursors,
                          // [20] ring overflow, [21] escalated sides, [22] block inspector queue,
-                         // [23] executor block queue
+                         // [23] executor block queue, [24] wide (ring-overflow) sides
     long long* totals;   // [0] words, [1] strips, [2] runs, [3] n_exec, [4] n_exec_block
     int* esc;            // escalated sides (inspector -> block inspector)
     long long* wl;       // executor words in list order (scratch)
     long long* wlo;      // exclusive scan of wl: pool offset of list position i
+    int* wide;           // sides whose band overflowed the regular ring (counters[24] of them)
 };
 
 struct Outputs {
@@ -62,25 +63,28 @@ cudaError_t launch_pack(const char* src, int64_t n, uint32_t* fwd, uint32_t* rev
 cudaError_t launch_validate_seeds(const long long* seeds, int n, int tlen, int qlen, long long* bad,
                                   cudaStream_t st);
 int inspector_blocks_per_sm(int R);
+// slist/nlist: inspect only the listed sides (nullptr: all 2n sides); listed sides are flagged SF_WIDE
 cudaError_t launch_inspect(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
-                           const SideArrays& sa, const ExecPlan& pl, int budget, cudaStream_t st);
+                           const SideArrays& sa, const ExecPlan& pl, int budget, const int* slist, int nlist,
+                           cudaStream_t st);
 cudaError_t launch_inspect_block(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
                                  const SideArrays& sa, const ExecPlan& pl, cudaStream_t st);
 int escalate_strips();  // FASTZ_ESCALATE_STRIPS (default 16; 0 disables block-per-side inspection)
 cudaError_t launch_census(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
-                          long long* cells, int* counter, cudaStream_t st);
+                          long long* cells, int* counter, const int* slist, int nlist, cudaStream_t st);
 cudaError_t launch_bin(int R, const DevParams& P, const SideArrays& sa, int nsides, const ExecPlan& pl, void* scan_tmp,
                        size_t scan_tmp_bytes, long long* tmp_a, long long* tmp_b, long long* tmp_c,
                        cudaStream_t st);
 size_t scan_tmp_bytes(int n);
+// list the sides flagged SF_WIDE (any order) and count them
+cudaError_t launch_wide_list(const SideArrays& sa, int nsides, int* list, int* count, cudaStream_t st);
 // redundant-alignment post-pass (dedup.cu; NEXT-3, reading R14)
 size_t redundant_tmp_bytes(int n);
 cudaError_t launch_redundant(void* recs, int n, void* tmp, size_t tmp_bytes, uint32_t* k1, uint32_t* k2, int* i1,
                              int* i2, int4* box, int2* sc, unsigned char* red, int* counters, cudaStream_t st);
 cudaError_t launch_execute(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
                            const SideArrays& sa, const ExecPlan& pl, int lo, int hi, int nblock, long long base,
-                           const Outputs& o,
-                           cudaStream_t st);
+                           const Outputs& o, int wide, cudaStream_t st);
 cudaError_t launch_traceback(int R, const SideArrays& sa, const ExecPlan& pl, int lo, int hi, int nblock,
                              long long base, const Outputs& o, cudaStream_t st);
 cudaError_t launch_combine_len(const DevParams& P, const Batch& b, const SideArrays& sa, const ExecPlan& pl,

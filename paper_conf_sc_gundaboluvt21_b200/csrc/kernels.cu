@@ -82,7 +82,11 @@ cudaError_t launch_validate_seeds(const long long* seeds, int n, int tlen, int q
 template <bool NM>
 __device__ __forceinline__ void setup_side(const Batch& b, int side, SideIO& io) {
     const int seed = side >> 1;
-    const long long tpos = b.seeds[2 * seed], qpos = b.seeds[2 * seed + 1];
+    long long tpos = b.seeds[2 * seed], qpos = b.seeds[2 * seed + 1];
+    // a seed outside [0, len] is reported by k_validate_seeds (FASTZ_ERANGE, the batch's results are void);
+    // until the host sees that flag its sides run as empty extensions at the origin, so no kernel ever reads
+    // outside the sequences
+    if (tpos < 0 || tpos > b.tlen || qpos < 0 || qpos > b.qlen) tpos = qpos = 0;
     if (side & 1) {
         io.Apk = b.Tf; io.Aoff = tpos; io.M = (int)(b.tlen - tpos);
         io.Bpk = b.Qf; io.Boff = qpos; io.Bmax = (int)(b.qlen - qpos);
@@ -194,7 +198,8 @@ __device__ __forceinline__ void write_side(const DevParams& P, const SideArrays&
 // A side still running after `budget` strips is handed to the block-per-side inspector (escalation).
 template <int R, bool NM>
 __device__ __forceinline__ void inspect_body(const DevParams& P, const Batch& b, int4* ring, int rmask,
-                                             const SideArrays& sa, const ExecPlan& pl, int budget) {
+                                             const SideArrays& sa, const ExecPlan& pl, int budget,
+                                             const int* __restrict__ slist, int nlist) {
     __shared__ SmemDP sm;
     smem_init<NM>(sm, P);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -202,15 +207,19 @@ __device__ __forceinline__ void inspect_body(const DevParams& P, const Batch& b,
     io_init(io, sm, ring, rmask, blockIdx.x * WARPS + warp, warp);
     io.eager_max = P.eager_max;
     io.budget = budget;
-    const int nsides = 2 * b.nseeds;
+    // slist: re-inspection of the sides whose band overflowed the regular ring (wide ring, SF_WIDE)
+    const int nsides = slist ? nlist : 2 * b.nseeds;
+    const uint32_t wide = slist ? SF_WIDE : 0u;
     for (;;) {
         int side = 0;
         if (lane == 0) side = atomicAdd(&pl.counters[0], 1);
         side = __shfl_sync(FULL, side, 0);
         if (side >= nsides) break;
+        if (slist) side = slist[side];
         setup_side<NM>(b, side, io);
         SideOut o;
         run_side<R, MODE_INSPECT, true, false, NM>(P, io, o);
+        o.flags |= wide;
         __syncwarp();  // eager corner codes (shared memory) written by lanes 0..4 -> read by lane 0
         if (lane == 0) {
             if (o.flags & SF_ESCALATE) {
@@ -236,16 +245,17 @@ __device__ __forceinline__ void inspect_body(const DevParams& P, const Batch& b,
 #endif
 template <int R>
 __global__ void INSPECT_ATTR k_inspect(DevParams P, Batch b, int4* ring, int rmask, SideArrays sa,
-                                                         ExecPlan pl, int budget) {
-    inspect_body<R, false>(P, b, ring, rmask, sa, pl, budget);
+                                                         ExecPlan pl, int budget, const int* slist, int nlist) {
+    inspect_body<R, false>(P, b, ring, rmask, sa, pl, budget, slist, nlist);
 }
 template <int R>
 #ifndef INSPECT_N_MAXREG
 #define INSPECT_N_MAXREG 80  // 6 CTAs per SM: measured 2% faster than 72 (which spills) on C2 with N runs
 #endif
 __global__ void __maxnreg__(INSPECT_N_MAXREG) k_inspect_n(DevParams P, Batch b, int4* ring, int rmask,
-                                                                           SideArrays sa, ExecPlan pl, int budget) {
-    inspect_body<R, true>(P, b, ring, rmask, sa, pl, budget);
+                                                                           SideArrays sa, ExecPlan pl, int budget,
+                                                                           const int* slist, int nlist) {
+    inspect_body<R, true>(P, b, ring, rmask, sa, pl, budget, slist, nlist);
 }
 
 // Block per side (long sides, escalated by k_inspect): the CTA's warps pipeline the side's strips.
@@ -279,18 +289,19 @@ __global__ void __launch_bounds__(WARPS * 32) k_inspect_block(DevParams P, Batch
 
 template <int R, bool NM>
 __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int4* ring, int rmask,
-                                                        long long* cells, int* counter) {
+                                                        long long* cells, int* counter, const int* slist, int nlist) {
     __shared__ SmemDP sm;
     smem_init<NM>(sm, P);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     SideIO io;
     io_init(io, sm, ring, rmask, blockIdx.x * WARPS + warp, warp);
-    const int nsides = 2 * b.nseeds;
+    const int nsides = slist ? nlist : 2 * b.nseeds;
     for (;;) {
         int side = 0;
         if (lane == 0) side = atomicAdd(counter, 1);
         side = __shfl_sync(FULL, side, 0);
         if (side >= nsides) break;
+        if (slist) side = slist[side];
         setup_side<NM>(b, side, io);
         SideOut o;
         run_side<R, MODE_CENSUS, false, false, NM>(P, io, o);
@@ -311,7 +322,8 @@ __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int
 template <int R, bool NM>
 __global__ void EXECUTE_ATTR k_execute(DevParams P, Batch b, int4* ring, int rmask,
                                                          SideArrays sa, ExecPlan pl, int lo, int hi, int nblock,
-                                                         long long base, Outputs out) {
+                                                         long long base, Outputs out, int wide) {
+    // wide = 1: this launch (the wide ring) runs only the SF_WIDE sides of the range, wide = 0 all others
     __shared__ SmemDP sm;
     __shared__ PipeShared ps;
     __shared__ int cur;
@@ -326,6 +338,10 @@ __global__ void EXECUTE_ATTR k_execute(DevParams P, Batch b, int4* ring, int rma
         __syncthreads();
         const int side = cur;
         if (side < 0) break;
+        if (((sa.flags[side] & SF_WIDE) != 0) != (wide != 0)) {
+            __syncthreads();  // cur is rewritten by thread 0 next iteration
+            continue;
+        }
         SideIO io;
         io_init(io, sm, ring, rmask, blockIdx.x * WARPS, warp);
         io.ps = &ps;
@@ -350,6 +366,7 @@ __global__ void EXECUTE_ATTR k_execute(DevParams P, Batch b, int4* ring, int rma
         idx = __shfl_sync(FULL, idx, 0);
         if (idx >= hi) break;
         const int side = pl.list[idx];
+        if (((sa.flags[side] & SF_WIDE) != 0) != (wide != 0)) continue;
         setup_side<NM>(b, side, io);
         if (!(P.options & OPT_NO_TRIM)) {
             io.M = sa.ti[side];
@@ -532,7 +549,10 @@ __global__ void k_bin_count(DevParams P, SideArrays sa, int nsides, ExecPlan pl,
     if (!skip && (P.options & OPT_NO_BINNING)) bin = 1;  // one queue, warp per side (ablation)
     pl.bin[s] = bin;
     atomicAdd(&pl.counters[2 + bin], 1);
-    if (fl & SF_RING) atomicOr(&pl.counters[20], 1);
+    if (fl & SF_RING) {  // band wider than the ring: re-inspected with a wider ring (api.cu)
+        atomicOr(&pl.counters[20], 1);
+        pl.wide[atomicAdd(&pl.counters[24], 1)] = s;
+    }
     const long long ns = sa.nstrip[s] >= 0 ? sa.nstrip[s] : ti / (32 * R) + 1;
     // bins >= bblock run block per side: strip s of the side owns words [s * maxsw, (s + 1) * maxsw)
     words[s] = skip ? 0 : (bin >= bblock ? ns * (long long)sa.maxsw[s] : sa.bound[s]);
@@ -579,6 +599,18 @@ __global__ void k_bin_scatter(ExecPlan pl, int nsides) {
     if (bin == 0) return;
     const int pos = atomicAdd(&pl.counters[10 + bin], 1);
     pl.list[pos] = s;
+}
+
+__global__ void k_wide_list(SideArrays sa, int nsides, int* list, int* count) {
+    const int s = blockIdx.x * blockDim.x + threadIdx.x;
+    if (s < nsides && (sa.flags[s] & SF_WIDE)) list[atomicAdd(count, 1)] = s;
+}
+
+cudaError_t launch_wide_list(const SideArrays& sa, int nsides, int* list, int* count, cudaStream_t st) {
+    cudaError_t e = cudaMemsetAsync(count, 0, 4, st);
+    if (e != cudaSuccess || nsides == 0) return e;
+    k_wide_list<<<(nsides + 255) / 256, 256, 0, st>>>(sa, nsides, list, count);
+    return cudaGetLastError();
 }
 
 int block_bin() {  // smallest executor bin run block per side (FASTZ_BLOCK_BIN, default 3: > 2048)
@@ -792,15 +824,16 @@ int escalate_strips() {  // read per call: tests and ablations switch it at run 
 
 
 cudaError_t launch_inspect(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
-                           const SideArrays& sa, const ExecPlan& pl, int budget, cudaStream_t st) {
+                           const SideArrays& sa, const ExecPlan& pl, int budget, const int* slist, int nlist,
+                           cudaStream_t st) {
     if (b.nseeds == 0) return cudaSuccess;
     const bool nm = b.TfN || b.QfN;
     if (R == 2) {
-        if (nm) k_inspect_n<2><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, pl, budget);
-        else k_inspect<2><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, pl, budget);
+        if (nm) k_inspect_n<2><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, pl, budget, slist, nlist);
+        else k_inspect<2><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, pl, budget, slist, nlist);
     } else {
-        if (nm) k_inspect_n<4><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, pl, budget);
-        else k_inspect<4><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, pl, budget);
+        if (nm) k_inspect_n<4><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, pl, budget, slist, nlist);
+        else k_inspect<4><<<grid, WARPS * 32, 0, st>>>(P, b, ring, rmask, sa, pl, budget, slist, nlist);
     }
     return cudaGetLastError();
 }
@@ -813,17 +846,17 @@ cudaError_t launch_inspect_block(int R, int grid, const DevParams& P, const Batc
 }
 
 cudaError_t launch_census(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
-                          long long* cells, int* counter, cudaStream_t st) {
+                          long long* cells, int* counter, const int* slist, int nlist, cudaStream_t st) {
     if (b.nseeds == 0) return cudaSuccess;
-    FZ_DISPATCH(k_census, grid, P, b, ring, rmask, cells, counter);
+    FZ_DISPATCH(k_census, grid, P, b, ring, rmask, cells, counter, slist, nlist);
     return cudaGetLastError();
 }
 
 cudaError_t launch_execute(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
                            const SideArrays& sa, const ExecPlan& pl, int lo, int hi, int nblock, long long base,
-                           const Outputs& o, cudaStream_t st) {
+                           const Outputs& o, int wide, cudaStream_t st) {
     if (hi <= lo) return cudaSuccess;
-    FZ_DISPATCH(k_execute, grid, P, b, ring, rmask, sa, pl, lo, hi, nblock, base, o);
+    FZ_DISPATCH(k_execute, grid, P, b, ring, rmask, sa, pl, lo, hi, nblock, base, o, wide);
     return cudaGetLastError();
 }
 

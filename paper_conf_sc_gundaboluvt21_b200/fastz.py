@@ -50,7 +50,9 @@ class fastz_stats(ctypes.Structure):
                 ("ms_combine", ctypes.c_float), ("n_warp_slots", ctypes.c_int32), ("n_seeds", ctypes.c_int64),
                 ("n_sides", ctypes.c_int64), ("n_eager_sides", ctypes.c_int64), ("n_exec_sides", ctypes.c_int64),
                 ("bin_counts", ctypes.c_int64 * 8), ("exec_words", ctypes.c_int64), ("cigar_bytes", ctypes.c_int64),
-                ("n_launches", ctypes.c_int64), ("n_waves", ctypes.c_int64), ("n_escalated", ctypes.c_int64)]
+                ("n_launches", ctypes.c_int64), ("n_waves", ctypes.c_int64), ("n_escalated", ctypes.c_int64),
+                ("n_wide_sides", ctypes.c_int64), ("exec_reserved_words", ctypes.c_int64),
+                ("n_selfcheck_fail", ctypes.c_int64)]
 
 
 class fastz_seed_params(ctypes.Structure):

@@ -144,9 +144,9 @@ def test_deterministic_repeat():
     assert np.array_equal(g1.rec, g2.rec) and g1.cigar == g2.cigar
 
 
-def test_unfolded_profile_large_scores():
-    """Scores too large to fold O+E into the int16 column profile (|sub + O + E| > 32767): the kernels take
-    the unfolded path (separate O+E add)."""
+def test_large_scores():
+    """Large scoring parameters (|sub| up to 24k, O + E = 8600, Y = 188000): substitution values with O + E
+    folded in stay exact in the kernels' int32 table and all scores stay far inside the int32 range."""
     hox = np.array([[91, -114, -31, -123], [-114, 100, -125, -31], [-31, -125, 100, -114], [-123, -31, -114, 91]])
     rng = random.Random(123)
     T = rseq(rng, 3000)
