@@ -47,7 +47,7 @@ def test_worked_two_sided(ex):
 
 @pytest.mark.parametrize("ex", GOLD["one_sided"], ids=lambda e: e["id"])
 def test_worked_one_sided_as_right_side(ex):
-    kw = {"ydrop": ex["ydrop"]} if "ydrop" in ex else {}
+    kw = {k: ex[k] for k in ("ydrop", "gap_open") if k in ex}
     bad, g, o, _ = compare(ex["A"], ex["B"], [(0, 0)], **kw)
     assert_ok(bad)
     assert int(g.rec[0]["right_score"]) == ex["score"]

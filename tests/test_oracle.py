@@ -60,7 +60,7 @@ def rand_params(rng):
 @pytest.mark.parametrize("ex", GOLD["one_sided"], ids=lambda e: e["id"])
 def test_worked_one_sided(ex):
     """E1-E6: e.g. E2 = 564 (GATTAC) - (O+E = 430, P:71-72) + 655 (GATTACA) = 789."""
-    p = dataclasses.replace(P0, ydrop=ex.get("ydrop", P0.ydrop))
+    p = dataclasses.replace(P0, ydrop=ex.get("ydrop", P0.ydrop), gap_open=ex.get("gap_open", P0.gap_open))
     s = core.one_sided(ex["A"], ex["B"], p)
     assert (s.score, s.i, s.j, s.ops) == (ex["score"], ex["i"], ex["j"], ex["ops"])
 
