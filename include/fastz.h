@@ -131,6 +131,28 @@ int fastz_create(const fastz_params *p, const char *target, int64_t tlen, const 
                  int device, void *cuda_stream, fastz_ctx **out);
 
 /*
+ * Packed input (multi-GPU broadcast of 2-bit sequences).  fastz_pack_sequence packs ASCII
+ * (ACGTNacgtn; host or device memory) of `len` bases into caller-owned DEVICE buffers: words[(len+15)/16]
+ * (16 bases per uint32, base k of a word in bits 2k+1:2k, A0 C1 G2 T3, an N packed as 0) and
+ * nmask[(len+15)/16] (bit k of a uint16 = base k is N).  revcomp = 1 packs the reverse complement.
+ * *has_n (may be NULL) = 1 if the sequence has an N.  Enqueued on `cuda_stream` (NULL = legacy default
+ * stream); synchronizes it.  EBASE reports the first invalid character's index; EINVAL for host words/nmask.
+ *
+ * fastz_create_packed creates a context exactly like fastz_create from such device buffers (t_nmask /
+ * q_nmask may be NULL: no N); the buffers are copied.  The context's query is the packed query as given
+ * (pack with revcomp = 1 for the minus strand; FASTZ_OPT_QUERY_REVCOMP is not applied again).
+ *
+ * fastz_get_packed exposes a context's packed forward copies (which = 0 target, 1 query) as device pointers
+ * valid until fastz_destroy (*nmask = NULL if the sequence has no N), e.g. as the source of a broadcast.
+ */
+int fastz_pack_sequence(const char *seq, int64_t len, int revcomp, uint32_t *words, uint16_t *nmask, int *has_n,
+                        int device, void *cuda_stream);
+int fastz_create_packed(const fastz_params *p, const uint32_t *t_words, const uint16_t *t_nmask, int64_t tlen,
+                        const uint32_t *q_words, const uint16_t *q_nmask, int64_t qlen, int device,
+                        void *cuda_stream, fastz_ctx **out);
+int fastz_get_packed(fastz_ctx *c, int which, const uint32_t **words, const uint16_t **nmask, int64_t *len);
+
+/*
  * Extend n seeds (host or device memory as `seeds_on_device` says; n may be 0).  Runs inspector, binning,
  * executor, traceback and CIGAR assembly on the context's stream; results stay on the device until
  * fastz_get_alignments.  Replaces the results of any previous call.  Errors: EINVAL, ERANGE (a seed out of

@@ -313,13 +313,16 @@ void fastz_destroy(fastz_ctx* c) {
     delete c;
 }
 
-int fastz_create(const fastz_params* p, const char* target, int64_t tlen, const char* query, int64_t qlen,
-                 int device, void* cuda_stream, fastz_ctx** out) {
+}  // extern "C"
+
+namespace {
+
+// context with parameters and stream, no sequences yet
+int ctx_begin(const fastz_params* p, int64_t tlen, int64_t qlen, int device, void* cuda_stream, fastz_ctx** out) {
     if (!out) return fail(FASTZ_EINVAL, "out is NULL");
     *out = nullptr;
     int r;
     if ((r = check_params(p))) return r;
-    if ((!target && tlen > 0) || (!query && qlen > 0)) return fail(FASTZ_EINVAL, "sequence pointer is NULL");
     if (tlen < 0 || qlen < 0 || tlen >= (1LL << 31) || qlen >= (1LL << 31))
         return fail(FASTZ_ERANGE, "sequence lengths must be in [0, 2^31)");
     CK(cudaSetDevice(device));
@@ -362,6 +365,77 @@ int fastz_create(const fastz_params* p, const char* target, int64_t tlen, const 
     c->dp.eager_max = p->eager_max;
     c->tlen = (int)tlen;
     c->qlen = (int)qlen;
+    *out = c;
+    return 0;
+}
+
+// launch geometry, boundary rings, events
+void ctx_finish(fastz_ctx* c) {
+    c->R = pick_R();
+    int sms = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, c->device);
+    c->grid = sms * inspector_blocks_per_sm(c->R);
+    c->nslots = c->grid * WARPS;
+    // per-warp boundary ring: the widest explored band is bounded by the query side length; capped (wider
+    // bands take the wide ring, fastz_extend_seeds)
+    int64_t want = std::max<int64_t>(std::max<int64_t>(c->tlen, c->qlen) + 64, 1024);
+    c->rmask = next_pow2(std::min<int64_t>(want, 1 << 15)) - 1;
+    if (const char* e = getenv("FASTZ_RING_ENTRIES"))  // tests: a small ring exercises the wide-band path
+        c->rmask = next_pow2(std::max<int64_t>(atoll(e), 64)) - 1;
+    for (auto& e : c->ev) cudaEventCreate(&e);
+    c->ev_ok = true;
+}
+
+// packed (2-bit words + N mask, device memory) -> the context's forward and reversed copies
+int upload_packed(fastz_ctx* c, const uint32_t* words, const uint16_t* nmask, int64_t len, DBuf& fwd, DBuf& rev,
+                  DBuf& fwdn, DBuf& revn, bool& has_n) {
+    const size_t words_n = (size_t)((len + 15) / 16) + 4;
+    const size_t used = (size_t)((len + 15) / 16);
+    int r;
+    if ((r = dalloc(c, fwd, words_n * 4))) return r;
+    if ((r = dalloc(c, rev, words_n * 4))) return r;
+    if ((r = dalloc(c, fwdn, words_n * 2))) return r;
+    if ((r = dalloc(c, revn, words_n * 2))) return r;
+    CK(cudaMemsetAsync(fwd.p, 0, words_n * 4, c->stream));
+    CK(cudaMemsetAsync(rev.p, 0, words_n * 4, c->stream));
+    CK(cudaMemsetAsync(fwdn.p, 0, words_n * 2, c->stream));
+    CK(cudaMemsetAsync(revn.p, 0, words_n * 2, c->stream));
+    has_n = false;
+    if (len == 0) return 0;
+    if (!is_device_ptr(words) || (nmask && !is_device_ptr(nmask)))
+        return fail(FASTZ_EINVAL, "packed sequences must be device memory");
+    CK(cudaMemcpyAsync(fwd.p, words, used * 4, cudaMemcpyDeviceToDevice, c->stream));
+    // bases past len in the last word must be 0 (the kernels read whole words)
+    if (len % 16) {
+        const uint32_t keep = (1u << (2 * (len % 16))) - 1u;
+        uint32_t last = 0;
+        CK(cudaMemcpyAsync(&last, words + used - 1, 4, cudaMemcpyDeviceToHost, c->stream));
+        CK(cudaStreamSynchronize(c->stream));
+        last &= keep;
+        CK(cudaMemcpyAsync(P_<uint32_t>(fwd) + used - 1, &last, 4, cudaMemcpyHostToDevice, c->stream));
+    }
+    if (nmask) CK(cudaMemcpyAsync(fwdn.p, nmask, used * 2, cudaMemcpyDeviceToDevice, c->stream));
+    if ((r = dalloc(c, c->small, 64))) return r;
+    CK(cudaMemsetAsync(c->small.p, 0, 4, c->stream));
+    CK(launch_reverse_packed(P_<uint32_t>(fwd), nmask ? P_<uint16_t>(fwdn) : nullptr, len, P_<uint32_t>(rev),
+                             P_<uint16_t>(revn), P_<int>(c->small), c->stream));
+    int hn = 0;
+    CK(cudaMemcpyAsync(&hn, c->small.p, 4, cudaMemcpyDeviceToHost, c->stream));
+    CK(cudaStreamSynchronize(c->stream));
+    has_n = hn != 0;
+    return 0;
+}
+
+}  // namespace
+
+extern "C" {
+
+int fastz_create(const fastz_params* p, const char* target, int64_t tlen, const char* query, int64_t qlen,
+                 int device, void* cuda_stream, fastz_ctx** out) {
+    if ((!target && tlen > 0) || (!query && qlen > 0)) return fail(FASTZ_EINVAL, "sequence pointer is NULL");
+    fastz_ctx* c = nullptr;
+    int r;
+    if ((r = ctx_begin(p, tlen, qlen, device, cuda_stream, &c))) return r;
     if ((r = upload_seq(c, target, tlen, c->Tf, c->Tr, c->TfN, c->TrN, c->t_has_n, 0, 0)) ||
         (r = upload_seq(c, query, qlen, c->Qf, c->Qr, c->QfN, c->QrN, c->q_has_n, tlen,
                         (p->options & FASTZ_OPT_QUERY_REVCOMP) ? 1 : 0))) {
@@ -369,19 +443,74 @@ int fastz_create(const fastz_params* p, const char* target, int64_t tlen, const 
         return r;
     }
     dfree(c, c->stage);
-    c->R = pick_R();
-    int sms = 0;
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-    c->grid = sms * inspector_blocks_per_sm(c->R);
-    c->nslots = c->grid * WARPS;
-    // per-warp boundary ring: the widest explored band is bounded by the query side length; capped
-    int64_t want = std::max<int64_t>(std::max<int64_t>(tlen, qlen) + 64, 1024);
-    c->rmask = next_pow2(std::min<int64_t>(want, 1 << 15)) - 1;
-    if (const char* e = getenv("FASTZ_RING_ENTRIES"))  // tests: a small ring exercises the wide-band path
-        c->rmask = next_pow2(std::max<int64_t>(atoll(e), 64)) - 1;
-    for (auto& e : c->ev) cudaEventCreate(&e);
-    c->ev_ok = true;
+    ctx_finish(c);
     *out = c;
+    return 0;
+}
+
+int fastz_create_packed(const fastz_params* p, const uint32_t* t_words, const uint16_t* t_nmask, int64_t tlen,
+                        const uint32_t* q_words, const uint16_t* q_nmask, int64_t qlen, int device, void* cuda_stream,
+                        fastz_ctx** out) {
+    if ((!t_words && tlen > 0) || (!q_words && qlen > 0)) return fail(FASTZ_EINVAL, "sequence pointer is NULL");
+    fastz_ctx* c = nullptr;
+    int r;
+    if ((r = ctx_begin(p, tlen, qlen, device, cuda_stream, &c))) return r;
+    if ((r = upload_packed(c, t_words, t_nmask, tlen, c->Tf, c->Tr, c->TfN, c->TrN, c->t_has_n)) ||
+        (r = upload_packed(c, q_words, q_nmask, qlen, c->Qf, c->Qr, c->QfN, c->QrN, c->q_has_n))) {
+        fastz_destroy(c);
+        return r;
+    }
+    ctx_finish(c);
+    *out = c;
+    return 0;
+}
+
+int fastz_pack_sequence(const char* seq, int64_t len, int revcomp, uint32_t* words, uint16_t* nmask, int* has_n,
+                        int device, void* cuda_stream) {
+    if ((!seq && len > 0) || (len > 0 && (!words || !nmask))) return fail(FASTZ_EINVAL, "NULL argument");
+    if (len < 0 || len >= (1LL << 31)) return fail(FASTZ_ERANGE, "length must be in [0, 2^31)");
+    CK(cudaSetDevice(device));
+    if (has_n) *has_n = 0;
+    if (len == 0) return 0;
+    if (!is_device_ptr(words) || !is_device_ptr(nmask)) return fail(FASTZ_EINVAL, "words/nmask must be device memory");
+    cudaStream_t st = (cudaStream_t)cuda_stream;
+    struct Scratch {  // released on every return path
+        void* p = nullptr;
+        cudaStream_t s = nullptr;
+        ~Scratch() {
+            if (s) cudaStreamSynchronize(s);
+            if (p) cudaFree(p);
+        }
+    } sc;
+    sc.s = st;
+    const char* dsrc = seq;
+    const size_t nw = (size_t)((len + 15) / 16);
+    const bool host = !is_device_ptr(seq);
+    CK(cudaMalloc(&sc.p, 64 + (host ? (size_t)len : 0) + nw * 8));
+    char* base = static_cast<char*>(sc.p);
+    long long* flags = reinterpret_cast<long long*>(base);
+    uint32_t* rev = reinterpret_cast<uint32_t*>(base + 64 + (host ? (size_t)len : 0));
+    uint16_t* revn = reinterpret_cast<uint16_t*>(rev + nw);
+    if (host) {
+        CK(cudaMemcpyAsync(base + 64, seq, (size_t)len, cudaMemcpyHostToDevice, st));
+        dsrc = base + 64;
+    }
+    long long init[2] = {LLONG_MAX, 0};
+    CK(cudaMemcpyAsync(flags, init, sizeof(init), cudaMemcpyHostToDevice, st));
+    CK(launch_pack(dsrc, len, words, rev, nmask, revn, flags, revcomp, st));
+    long long res[2] = {0, 0};
+    CK(cudaMemcpyAsync(res, flags, sizeof(res), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (res[0] != LLONG_MAX) return fail(FASTZ_EBASE, "invalid base character at index " + std::to_string(res[0]));
+    if (has_n) *has_n = res[1] != 0;
+    return 0;
+}
+
+int fastz_get_packed(fastz_ctx* c, int which, const uint32_t** words, const uint16_t** nmask, int64_t* len) {
+    if (!c || (which != 0 && which != 1)) return fail(FASTZ_EINVAL, "bad argument");
+    if (words) *words = P_<uint32_t>(which ? c->Qf : c->Tf);
+    if (nmask) *nmask = (which ? c->q_has_n : c->t_has_n) ? P_<uint16_t>(which ? c->QfN : c->TfN) : nullptr;
+    if (len) *len = which ? c->qlen : c->tlen;
     return 0;
 }
 
@@ -741,7 +870,7 @@ int fastz_mark_redundant_records(fastz_alignment* recs, int64_t n, int recs_on_d
             if (s) cudaStreamDestroy(s);
         }
     } sc;
-    CK(cudaStreamCreateWithFlags(&sc.s, cudaStreamNonBlocking));
+    CK(cudaStreamCreateWithFlags(&sc.s, cudaStreamDefault));  // ordered after the legacy default stream
     const size_t m = (size_t)n;
     auto up = [](size_t b) { return (b + 255) & ~(size_t)255; };
     const size_t tb = redundant_tmp_bytes((int)n);

@@ -60,6 +60,8 @@ int pick_R();  // rows per lane (FASTZ_R env: 2, 4 or 8; default 4)
 
 cudaError_t launch_pack(const char* src, int64_t n, uint32_t* fwd, uint32_t* rev, uint16_t* fwdn, uint16_t* revn,
                         long long* bad, int revcomp, cudaStream_t st);
+cudaError_t launch_reverse_packed(const uint32_t* fwd, const uint16_t* fwdn, int64_t n, uint32_t* rev, uint16_t* revn,
+                                  int* has_n, cudaStream_t st);
 cudaError_t launch_validate_seeds(const long long* seeds, int n, int tlen, int qlen, long long* bad,
                                   cudaStream_t st);
 int inspector_blocks_per_sm(int R);

@@ -62,6 +62,35 @@ cudaError_t launch_pack(const char* src, int64_t n, uint32_t* fwd, uint32_t* rev
     return cudaGetLastError();
 }
 
+// Reversed copy (and N mask) of a packed sequence: base p of the output is base n-1-p of the input.  Also ORs
+// every input mask word into *has_n.  One thread per output word of 16 bases.
+__global__ void k_reverse_packed(const uint32_t* __restrict__ fwd, const uint16_t* __restrict__ fwdn, long long n,
+                                 uint32_t* __restrict__ rev, uint16_t* __restrict__ revn, int* has_n) {
+    const long long w = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    const long long nw = (n + 15) / 16;
+    if (w >= nw) return;
+    uint32_t r = 0, rn = 0;
+    for (int i = 0; i < 16; ++i) {
+        const long long p = 16 * w + i;
+        if (p < n) {
+            const long long q = n - 1 - p;
+            r |= ((fwd[q >> 4] >> (2 * (q & 15))) & 3u) << (2 * i);
+            if (fwdn) rn |= ((uint32_t)(fwdn[q >> 4] >> (q & 15)) & 1u) << i;
+        }
+    }
+    rev[w] = r;
+    revn[w] = (uint16_t)rn;
+    if (fwdn && fwdn[w]) atomicOr(has_n, 1);
+}
+
+cudaError_t launch_reverse_packed(const uint32_t* fwd, const uint16_t* fwdn, int64_t n, uint32_t* rev, uint16_t* revn,
+                                  int* has_n, cudaStream_t st) {
+    const long long nw = (n + 15) / 16;
+    if (nw == 0) return cudaSuccess;
+    k_reverse_packed<<<(unsigned)((nw + 255) / 256), 256, 0, st>>>(fwd, fwdn, n, rev, revn, has_n);
+    return cudaGetLastError();
+}
+
 __global__ void k_validate_seeds(const long long* __restrict__ seeds, int n, int tlen, int qlen, long long* bad) {
     const int s = blockIdx.x * blockDim.x + threadIdx.x;
     if (s >= n) return;

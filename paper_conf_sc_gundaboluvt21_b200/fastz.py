@@ -26,7 +26,8 @@ OPT_NO_EAGER, OPT_NO_TRIM, OPT_NO_BINNING, OPT_NO_BLOCK, OPT_TRACEBACK_ABOVE_K =
 EXPORTS = ["fastz_default_params", "fastz_create", "fastz_extend_seeds", "fastz_get_alignments",
            "fastz_get_alignments_device", "fastz_get_sides", "fastz_census", "fastz_get_stats",
            "fastz_destroy", "fastz_strerror", "fastz_int_peak", "fastz_default_seed_params", "fastz_find_hsps",
-           "fastz_mark_redundant", "fastz_mark_redundant_records"]
+           "fastz_mark_redundant", "fastz_mark_redundant_records", "fastz_pack_sequence", "fastz_create_packed",
+           "fastz_get_packed"]
 
 
 class FastzError(RuntimeError):
@@ -102,7 +103,12 @@ def lib() -> ctypes.CDLL:
     L.fastz_default_seed_params.restype = None
     L.fastz_find_hsps.argtypes = [vp, ctypes.POINTER(fastz_seed_params), vp, vp, i64, ctypes.POINTER(i64),
                                   ctypes.POINTER(i64)]
-    for name in ("fastz_find_hsps", "fastz_create", "fastz_extend_seeds", "fastz_get_alignments", "fastz_get_alignments_device",
+    L.fastz_pack_sequence.argtypes = [vp, i64, i32, vp, vp, ctypes.POINTER(i32), i32, vp]
+    L.fastz_create_packed.argtypes = [ctypes.POINTER(fastz_params), vp, vp, i64, vp, vp, i64, i32, vp,
+                                      ctypes.POINTER(vp)]
+    L.fastz_get_packed.argtypes = [vp, i32, ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.POINTER(i64)]
+    for name in ("fastz_pack_sequence", "fastz_create_packed", "fastz_get_packed", "fastz_mark_redundant",
+                 "fastz_mark_redundant_records", "fastz_find_hsps", "fastz_create", "fastz_extend_seeds", "fastz_get_alignments", "fastz_get_alignments_device",
                  "fastz_get_sides", "fastz_census", "fastz_get_stats", "fastz_int_peak"):
         getattr(L, name).restype = i32
     _lib = L
@@ -156,6 +162,32 @@ def fastz_create(params: fastz_params, target, query, device: int = 0, stream: i
     return out.value
 
 
+def fastz_pack_sequence(seq, revcomp: bool = False, device: int = 0, stream: int | None = None):
+    """ASCII (bytes / numpy / torch, host or device) -> (words int32 tensor, nmask int16 tensor, has_n) on
+    cuda:device, as fastz_pack_sequence writes them (2-bit codes, 16 per word; 1-bit N mask)."""
+    import torch
+    sp, sl, _, keep = _ptr_len(seq)
+    nw = (sl + 15) // 16
+    dev = torch.device("cuda", device)
+    words = torch.zeros(max(nw, 1), dtype=torch.int32, device=dev)
+    nmask = torch.zeros(max(nw, 1), dtype=torch.int16, device=dev)
+    has_n = ctypes.c_int32()
+    _check(lib().fastz_pack_sequence(sp, sl, 1 if revcomp else 0, words.data_ptr(), nmask.data_ptr(),
+                                     ctypes.byref(has_n), device, stream))
+    del keep
+    return words[:nw], nmask[:nw], bool(has_n.value)
+
+
+def fastz_create_packed(params: fastz_params, t_words, t_nmask, tlen: int, q_words, q_nmask, qlen: int,
+                        device: int = 0, stream: int | None = None) -> int:
+    """Context from packed device tensors (``fastz_pack_sequence`` layout); a mask may be None (no N)."""
+    out = ctypes.c_void_p()
+    ptr = lambda t: None if t is None else t.data_ptr()  # noqa: E731
+    _check(lib().fastz_create_packed(ctypes.byref(params), ptr(t_words), ptr(t_nmask), int(tlen), ptr(q_words),
+                                     ptr(q_nmask), int(qlen), device, stream, ctypes.byref(out)))
+    return out.value
+
+
 def fastz_extend_seeds(ctx: int, seeds) -> int:
     """seeds: (n, 2) int64 cut points as numpy (host) or a CUDA torch tensor (device)."""
     try:
@@ -180,6 +212,30 @@ def fastz_get_alignments(ctx: int):
     cig = ctypes.create_string_buffer(max(nb.value, 1))
     _check(lib().fastz_get_alignments(ctx, rec.ctypes.data, n.value, cig, nb.value, ctypes.byref(n), ctypes.byref(nb)))
     return rec[:n.value], cig.raw[:nb.value]
+
+
+class _DevView:
+    """__cuda_array_interface__ over library-owned device memory (zero-copy torch.as_tensor)."""
+
+    def __init__(self, ptr: int, nbytes: int):
+        self.__cuda_array_interface__ = {"shape": (nbytes,), "typestr": "|u1", "data": (ptr or 0, True),
+                                         "version": 3, "strides": None}
+
+
+def fastz_get_alignments_device(ctx: int, device: int = 0):
+    """(records uint8[n, 64], cigar uint8[bytes]) as torch tensors ALIASING the context's device memory (valid
+    until the next extend / destroy).  The caller must order its reads after the context's stream."""
+    import torch
+    recs, cig = ctypes.c_void_p(), ctypes.c_void_p()
+    n, nb = ctypes.c_int64(), ctypes.c_int64()
+    _check(lib().fastz_get_alignments_device(ctx, ctypes.byref(recs), ctypes.byref(cig), ctypes.byref(n),
+                                             ctypes.byref(nb)))
+    dev = torch.device("cuda", device)
+    r = torch.as_tensor(_DevView(recs.value, n.value * 64), device=dev).view(n.value, 64) if n.value else \
+        torch.zeros((0, 64), dtype=torch.uint8, device=dev)
+    c = torch.as_tensor(_DevView(cig.value, nb.value), device=dev) if nb.value else \
+        torch.zeros(0, dtype=torch.uint8, device=dev)
+    return r, c
 
 
 def fastz_get_sides(ctx: int, n: int):
@@ -216,6 +272,18 @@ def fastz_mark_redundant_records(rec: np.ndarray, device: int = 0):
     _check(lib().fastz_mark_redundant_records(rec.ctypes.data if n else None, n, 0, red.ctypes.data,
                                               ctypes.byref(cnt), device))
     return red[:n], cnt.value
+
+
+def fastz_mark_redundant_records_device(rec, device: int = 0) -> int:
+    """Context-free post-pass (reading R14) on DEVICE records (a contiguous CUDA tensor holding n x 64-byte
+    fastz_alignment records): sets FLAG_REDUNDANT in place; returns the count.  Orders itself after the
+    current PyTorch stream."""
+    import torch
+    n = rec.numel() // ALIGN_DTYPE.itemsize
+    torch.cuda.current_stream(rec.device).synchronize()
+    cnt = ctypes.c_int64()
+    _check(lib().fastz_mark_redundant_records(rec.data_ptr() if n else None, n, 1, None, ctypes.byref(cnt), device))
+    return cnt.value
 
 
 def fastz_get_stats(ctx: int) -> dict:
@@ -287,6 +355,20 @@ def torch_allocator_hooks(device: int = 0):
 # ----------------------------------------------------------------------------------- convenience class
 
 @dataclass
+class PackedSequence:
+    """A 2-bit packed sequence on the device (``fastz_pack_sequence`` layout); nmask None = no N."""
+    words: object
+    nmask: object
+    length: int
+
+    @staticmethod
+    def pack(seq, revcomp: bool = False, device: int = 0, stream: int | None = None) -> "PackedSequence":
+        w, m, has_n = fastz_pack_sequence(seq, revcomp, device, stream)
+        n = len(seq) if not hasattr(seq, "numel") else seq.numel()
+        return PackedSequence(w, m if has_n else None, int(n))
+
+
+@dataclass
 class Alignments:
     rec: np.ndarray
     cigar: bytes = field(repr=False)
@@ -316,10 +398,25 @@ class Aligner:
                     stream = torch.cuda.current_stream(device).cuda_stream
             except ImportError:  # pragma: no cover
                 stream = None
-        self.ctx = fastz_create(self.params, target, query, device, stream)
+        self.device = device
+        self.stream = stream
+        if isinstance(target, PackedSequence):
+            self.ctx = fastz_create_packed(self.params, target.words, target.nmask, target.length, query.words,
+                                           query.nmask, query.length, device, stream)
+        else:
+            self.ctx = fastz_create(self.params, target, query, device, stream)
         self.n = 0
 
     def extend_only(self, seeds) -> int:
+        try:
+            import torch
+            if isinstance(seeds, torch.Tensor) and seeds.is_cuda:
+                seeds = seeds.to(torch.int64).contiguous()
+                cur = torch.cuda.current_stream(seeds.device)
+                if cur.cuda_stream != (self.stream or 0):
+                    cur.synchronize()  # the seeds were produced on another stream than the context's
+        except ImportError:  # pragma: no cover
+            pass
         self.n = fastz_extend_seeds(self.ctx, seeds)
         return self.n
 
@@ -327,6 +424,17 @@ class Aligner:
         self.extend_only(seeds)
         rec, cig = fastz_get_alignments(self.ctx)
         return Alignments(rec, cig)
+
+    def results_device(self):
+        """(records uint8[n, 64], cigar uint8[bytes]) torch tensors aliasing the context's device memory, with the
+        context's stream synchronized (so any stream may read them)."""
+        import torch
+        r, c = fastz_get_alignments_device(self.ctx, self.device)
+        if self.stream:
+            torch.cuda.ExternalStream(self.stream, device=torch.device("cuda", self.device)).synchronize()
+        else:
+            torch.cuda.synchronize(self.device)
+        return r, c
 
     def results(self) -> Alignments:
         rec, cig = fastz_get_alignments(self.ctx)

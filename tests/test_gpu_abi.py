@@ -120,3 +120,30 @@ def test_torch_caching_allocator_hooks():
     with fastz.Aligner(w.T, w.Q, torch_alloc=True) as c:   # reuses the cached blocks
         rc = c.extend(w.seeds)
     assert np.array_equal(ra.rec, rc.rec)
+
+
+def test_packed_contexts_equal_ascii_contexts():
+    """fastz_pack_sequence + fastz_create_packed (the multi-GPU broadcast format) give the same results as
+    fastz_create from ASCII: plain, with N bases (masks), and the minus strand (revcomp packing)."""
+    w = _w()
+    T = bytearray(w.T)
+    T[100:130] = b"N" * 30
+    T = bytes(T)
+    for tq, opts in (((w.T, w.Q), 0), ((T, w.Q.lower()), 0), ((w.T, w.Q), fastz.OPT_QUERY_REVCOMP)):
+        with fastz.Aligner(tq[0], tq[1], fastz.fastz_default_params(options=opts)) as a:
+            ra = a.extend(w.seeds)
+        pt = fastz.PackedSequence.pack(tq[0])
+        pq = fastz.PackedSequence.pack(tq[1], revcomp=bool(opts & fastz.OPT_QUERY_REVCOMP))
+        assert (pt.nmask is not None) == (b"N" in tq[0])
+        with fastz.Aligner(pt, pq) as b:
+            rb = b.extend(w.seeds)
+            rd, cd = b.results_device()
+            assert rd.shape == (len(w.seeds), 64) and cd.numel() == len(rb.cigar)
+            assert rd.cpu().numpy().tobytes() == rb.rec.tobytes() and cd.cpu().numpy().tobytes() == rb.cigar
+        assert np.array_equal(ra.rec, rb.rec) and ra.cigar == rb.cigar
+
+
+def test_pack_sequence_rejects_invalid_base():
+    with pytest.raises(fastz.FastzError) as e:
+        fastz.fastz_pack_sequence(b"ACGTACGTACGTACGTACGX")
+    assert e.value.status == fastz.FASTZ_EBASE and "index 19" in str(e.value)
