@@ -1,17 +1,24 @@
 #!/usr/bin/env python
 """Benchmark of the FastZ hot path on B200 (driver contract: one JSON line on rank 0).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--config 2] [--impl fastz|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config 3] [--impl fastz|reference]
 
-Workload (BASELINE.json configs[1], "C2"): synthetic 10 Mbp chromosome pair, 2^20 seeds per GPU with the
-paper's skewed extension-length mix (synth.genome.config2).  One step = one call
-of fastz_extend_seeds over the whole seed batch: inspector + eager traceback, binning, trimmed executor,
-traceback and CIGAR assembly, with the seeds and sequences already resident in HBM (``value``); ``e2e``
-repeats it through the public API from pinned host seeds to host records + CIGAR text.
+Headline workload (BASELINE.json configs[2], "C3", the largest single-GPU config): synthetic 100 Mbp
+chromosome-scale pair, 2^21 seeds per GPU, with 16-64 kbp high-scoring alignments among the paper's skewed
+length mix (synth.genome.config3).  One step = one fastz_extend_seeds call over the
+whole seed batch: inspector + eager traceback, binning, trimmed executor, traceback and CIGAR assembly, seeds
+and sequences resident in HBM (``value``); ``e2e`` repeats it through the public API from pinned host seeds to
+host records + CIGAR text.  ``secondary`` holds the same measurement on C2 (10 Mbp, 2^20 seeds).
+
+``genome_pair`` (whole-genome-pair wall time on C4, 2^30 bp x 2^30 bp, 2^23 seeds): the
+multi-GPU driver ``dist.extend_genome_pair`` over all N ranks -- rank 0 packs and broadcasts the sequences
+(2 bits per base) and the seeds, every rank extends its hash shard, records are gathered to rank 0 over NCCL and
+put back in seed order, results end on rank 0's host; max over ranks of the device-synchronised wall clock.
 
 Metric: GCUPS = explored DP cells (origin + cells with a live neighbour, reading R7 -- the exact
 count, produced once by the census kernel and parity-tested against the oracle) / step time.  Multi-GPU:
-seeds are sharded, nothing is exchanged in the timed region (scaling "weak"); time = max over ranks.
+each rank extends its own 2^21-seed shard of the same pair, nothing is exchanged in the timed region (scaling
+"weak"); time = max over ranks.
 
 --impl reference times the CPU oracle (oracle/, the plain sequential implementation) on a bounded sample
 of the same workload on this box's host cores; it is the reference arm of this tier.
@@ -30,7 +37,12 @@ import time
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
-OPS_PER_CELL = 13  # 9 recurrence ops (4 max + 5 add) + 4 cone y-drop ops
+# algorithmic integer ops per explored cell: the recurrences' 4 max + 5 add.
+# The cone y-drop adds 4 more (2 max, 1 add, 1 compare), reported separately as frac_with_ydrop.
+OPS_PER_CELL = 9
+OPS_PER_CELL_YDROP = 13
+PAPER_CONTEXT = {"fastz_rtx3080_vs_sequential_lastz": 111, "multicore_lastz_16c_vs_sequential": 20,
+                 "source": "PAPER.md P:22, P:279-281 (context only: different baseline program and hardware)"}
 
 
 def parse():
@@ -38,11 +50,13 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", type=int, default=2)
+    ap.add_argument("--config", type=int, default=3)
     ap.add_argument("--seeds", type=int, default=0, help="seeds per GPU (default: the config's)")
     ap.add_argument("--impl", default="fastz", choices=["fastz", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--profile", action="store_true", help="one warm-up + 1 step, for ncu")
+    ap.add_argument("--no-secondary", action="store_true", help="skip the C2 secondary measurement")
+    ap.add_argument("--no-genome-pair", action="store_true", help="skip the C4 genome-pair wall time")
+    ap.add_argument("--profile", action="store_true", help="one warm-up + 1 step of the headline only, for ncu")
     return ap.parse_args()
 
 
@@ -53,32 +67,24 @@ def dist_env():
     return ws, rank, local
 
 
+DESC = {
+    1: "C1: synthetic 100 kbp target vs mutated copy (~10% subs, 1% indels), 2,048 seeds",
+    2: "C2: synthetic 10 Mbp chromosome pair, 2^20 seeds per GPU, skewed extension lengths (>97% <=128 bp)",
+    3: "C3: synthetic 100 Mbp chromosome-scale pair, 2^21 seeds per GPU, long (16-64 kbp) high-scoring alignments",
+    5: "C5: extension-length stress sweep 32 bp - 64 kbp, 2^20 seeds per GPU",
+    6: "C6 (NEXT-2): dissimilar 10 Mbp pair, diverged short homology (cross-genus analog, P:331-340)",
+}
+DEFAULT_SEEDS = {1: 2048, 2: 1 << 20, 3: 1 << 21, 5: 1 << 20, 6: 1 << 20}
+
+
 def workload(config: int, n_per_gpu: int, world: int, rank: int):
     from synth import genome
-    if config == 2:
-        n = n_per_gpu or (1 << 20)
-        w = genome.config2(n_seeds=n * world)
-        desc = "C2: synthetic 10 Mbp chromosome pair, skewed extension lengths (>97% <=128 bp), LASTZ default scoring"
-    elif config == 1:
-        n = n_per_gpu or 2048
-        w = genome.config1(n_seeds=n * world)
-        desc = "C1: synthetic 100 kbp target vs mutated copy (~10% subs, 1% indels)"
-    elif config == 5:
-        n = n_per_gpu or (1 << 20)
-        w = genome.config5(n_seeds=n * world)
-        desc = "C5: extension-length stress sweep 32 bp - 64 kbp"
-    elif config == 6:
-        n = n_per_gpu or (1 << 20)
-        w = genome.config6(n_seeds=n * world)
-        desc = "C6 (NEXT-2): dissimilar 10 Mbp pair, diverged short homology (cross-genus analog, P:331-340)"
-    elif config == 3:
-        n = n_per_gpu or (1 << 21)
-        w = genome.config3(n_seeds=n * world)
-        desc = "C3: synthetic 100 Mbp pair with 16-64 kbp alignments"
-    else:
+    if config not in DESC:
         raise SystemExit(f"config {config} not supported by bench")
+    n = n_per_gpu or DEFAULT_SEEDS[config]
+    w = genome.make(config, n_seeds=n * world)
     shard = w.seeds[rank::world][:n]
-    return w, shard, desc
+    return w, shard, DESC[config]
 
 
 class Clocks:
@@ -120,28 +126,63 @@ class Clocks:
                 "reasons": sorted(reasons), "samples": len(rows)}
 
 
-def cpu_baseline(w, seeds, target_s=15.0):
-    """The oracle as it stands on this box's host cores, on a bounded random sample of the workload."""
-    import numpy as np
-    from oracle import core
+def host_cpu():
+    """CPU model, clock and usable cores of this host (lscpu / /proc/cpuinfo)."""
     cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count()
-    rng = np.random.default_rng(12345)
-    n = min(len(seeds), max(64, 8 * cores))
-    idx = rng.choice(len(seeds), n, replace=False)
-    t0 = time.perf_counter()
-    r = core.extend(w.T, w.Q, seeds[idx], threads=cores)
-    dt = time.perf_counter() - t0
-    if dt < target_s / 3 and n < len(seeds):
-        n2 = min(len(seeds), int(n * target_s / max(dt, 1e-3)))
-        idx = rng.choice(len(seeds), n2, replace=False)
+    model, mhz = None, None
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            k, _, v = line.partition(":")
+            if k.strip() == "Model name":
+                model = v.strip()
+            elif k.strip() in ("CPU max MHz", "CPU MHz") and mhz is None:
+                mhz = float(v.strip())
+    except Exception:
+        pass
+    if mhz is None:
+        try:
+            for line in open("/proc/cpuinfo"):
+                if line.startswith("cpu MHz"):
+                    mhz = float(line.split(":")[1])
+                    break
+        except Exception:
+            pass
+    return {"model": model, "mhz": mhz, "cores": cores}
+
+
+def _oracle_rate(w, seeds, threads, target_s, rng):
+    """Oracle cells/s on a random sample of ``seeds`` sized for about ``target_s`` seconds."""
+    from oracle import core
+    n = min(len(seeds), max(16, 4 * threads))
+    for _ in range(4):
+        idx = rng.choice(len(seeds), n, replace=False)
         t0 = time.perf_counter()
-        r = core.extend(w.T, w.Q, seeds[idx], threads=cores)
+        r = core.extend(w.T, w.Q, seeds[idx], threads=threads)
         dt = time.perf_counter() - t0
-        n = n2
+        if dt >= target_s / 3 or n >= len(seeds):
+            break
+        n = min(len(seeds), int(n * target_s / max(dt, 1e-3)))
     cells = int(r.rec["l_explored"].sum() + r.rec["r_explored"].sum())
-    return {"value": cells / dt / 1e9, "unit": "GCUPS", "cores": cores, "kind": "oracle",
-            "sample": f"{n} random seeds of the same workload ({cells} explored cells) in {dt:.2f} s, "
-                      f"{cores} threads", "seeds_per_s": n / dt}
+    return cells / dt, n, cells, dt
+
+
+def cpu_baseline(w, seeds, gpu_gcups):
+    """The oracle as it stands on this box's host cores (all of them, and one), on bounded random samples of
+    the same workload; GPU speed-ups beside the paper's (context)."""
+    import numpy as np
+    cpu = host_cpu()
+    rng = np.random.default_rng(12345)
+    rate_all, n_all, cells_all, dt_all = _oracle_rate(w, seeds, cpu["cores"], 15.0, rng)
+    rate_1, n_1, cells_1, dt_1 = _oracle_rate(w, seeds, 1, 6.0, rng)
+    return {"value": rate_all / 1e9, "unit": "GCUPS", "cores": cpu["cores"], "kind": "oracle",
+            "sample": f"{n_all} random seeds of the same workload ({cells_all} explored cells) in {dt_all:.2f} s on "
+                      f"{cpu['cores']} threads; 1-thread rate from {n_1} seeds ({cells_1} cells) in {dt_1:.2f} s",
+            "cpu_model": cpu["model"], "cpu_mhz": cpu["mhz"],
+            "one_core_gcups": rate_1 / 1e9, "seeds_per_s": n_all / dt_all,
+            "gpu_speedup_vs_all_cores": gpu_gcups / (rate_all / 1e9),
+            "gpu_speedup_vs_one_core": gpu_gcups / (rate_1 / 1e9),
+            "paper_context": PAPER_CONTEXT}
 
 
 def run_reference(args, ws, rank):
@@ -150,7 +191,8 @@ def run_reference(args, ws, rank):
     import numpy as np
     from oracle import core
     w, seeds, desc = workload(args.config, args.seeds, 1, 0)
-    cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count()
+    cpu = host_cpu()
+    cores = cpu["cores"]
     rng = np.random.default_rng(777)
     per = max(64, 6 * cores)
     # calibrate so one step takes ~8 s on this host
@@ -173,9 +215,88 @@ def run_reference(args, ws, rank):
             "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
             "config": {"workload": desc, "seeds_per_step": per, "sample": "random seeds of the workload per step"},
             "cpu_baseline": {"value": v, "unit": "GCUPS", "cores": cores, "kind": "oracle",
+                             "cpu_model": cpu["model"], "cpu_mhz": cpu["mhz"],
                              "sample": f"{per} random seeds per step x {args.steps} steps"},
             "e2e": {"value": v, "unit": "GCUPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+def measure(al, seeds_d, steps, warmup, stream, flush, ws, clocks=None):
+    """Device-timed steps (CUDA events on the library's stream, L2 flushed between steps, untimed)."""
+    import torch
+    import torch.distributed as dist
+    for _ in range(warmup):
+        al.extend_only(seeds_d)
+    torch.cuda.synchronize()
+    if ws > 1:
+        dist.barrier()
+    clk = clocks() if clocks else None
+    times, stages, launches = [], [], 0
+    for _ in range(steps):
+        flush.zero_()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        e0.record(stream)
+        al.extend_only(seeds_d)
+        e1.record(stream)
+        e1.synchronize()
+        times.append(e0.elapsed_time(e1))
+        s = al.stats()
+        stages.append(s)
+        launches += int(s["n_launches"])
+    torch.cuda.synchronize()
+    clk_rec = clk.stop() if clk else None
+    if ws > 1:
+        dist.barrier()
+    return times, stages, launches, clk_rec
+
+
+def genome_pair(ws, rank, local):
+    """C4 whole-genome-pair wall time through dist.extend_genome_pair on all ranks (rank 0's host ASCII + seeds
+    -> rank 0's host records + CIGARs); first (cold: context + pool allocation) and second (warm) run."""
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_gundaboluvt21_b200 import dist as fzdist
+    w = None
+    t_gen = 0.0
+    if rank == 0:
+        from synth import genome
+        t0 = time.perf_counter()
+        w = genome.config4()
+        t_gen = time.perf_counter() - t0
+    runs = []
+    for _ in range(2):
+        torch.cuda.synchronize()
+        if ws > 1:
+            dist.barrier()
+        tm = {}
+        t0 = time.perf_counter()
+        rec, cig = fzdist.extend_genome_pair(w.T if w else None, w.Q if w else None, w.seeds if w else None,
+                                             timings=tm, torch_alloc=True)
+        torch.cuda.synchronize()
+        dt = time.perf_counter() - t0
+        t = torch.tensor([dt, tm["broadcast_s"], tm["extend_s"], tm["gather_s"]], dtype=torch.float64,
+                         device=torch.device("cuda", local))
+        if ws > 1:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        runs.append([float(x) for x in t.tolist()])
+        if rank == 0:
+            n = len(rec)
+            cbytes = len(cig)
+        del rec, cig
+    if rank != 0:
+        return None
+    cold, warm = runs
+    return {"workload": "C4: synthetic 2^30 bp x 2^30 bp genome pair, 2^23 seeds (C2 block mix x100), LASTZ default "
+                        "scoring", "n_gpus": ws, "seeds": n, "cigar_bytes": cbytes,
+            "wall_s": warm[0], "cold_wall_s": cold[0],
+            "phases_s_max_over_ranks": {"broadcast": warm[1], "extend": warm[2], "gather_merge_d2h": warm[3]},
+            "seed_extensions_per_s": n / warm[0],
+            "timing": "time.perf_counter around extend_genome_pair after a barrier and device sync, max over ranks; "
+                      "2-bit sequence broadcast, extension, NCCL gather + seed-order merge, copy to rank 0's host "
+                      "included; seed finding and input generation excluded",
+            "generation_s": t_gen}
 
 
 def run_fastz(args, ws, rank, local):
@@ -200,32 +321,16 @@ def run_fastz(args, ws, rank, local):
     peak_ops, peak_mhz = fastz.fastz_int_peak(local, 300.0)
 
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
-    for _ in range(args.warmup):
-        al.extend_only(seeds_d)
-    torch.cuda.synchronize()
-    if ws > 1:
-        dist.barrier()
-    clk = Clocks(local)
-    times, insp, stages = [], [], []
-    launches = 0
-    for _ in range(args.steps):
-        flush.zero_()  # L2 flushed between timed steps (outside the events)
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        torch.cuda.synchronize()
-        e0.record(stream)
-        al.extend_only(seeds_d)
-        e1.record(stream)
-        e1.synchronize()
-        times.append(e0.elapsed_time(e1))
-        s = al.stats()
-        insp.append(s["ms_inspect"])
-        stages.append(s)
-        launches += int(s["n_launches"])
-    torch.cuda.synchronize()
-    clocks = clk.stop()
-    if ws > 1:
-        dist.barrier()
+    if args.profile:
+        args.warmup, args.steps = 1, 1
+    times, stages, launches, clocks = measure(al, seeds_d, args.steps, args.warmup, stream, flush, ws,
+                                              clocks=lambda: Clocks(local))
     ms = sum(times) / len(times)
+    if args.profile:
+        al.close()
+        if rank == 0:
+            print(json.dumps({"profile": True, "ms_per_step": ms}), flush=True)
+        return
 
     # e2e through the public API: pinned host seeds -> host records + CIGAR (the Aligner's page-locked result
     # buffers are allocated once, untimed, as a long-running user would keep them)
@@ -243,57 +348,58 @@ def run_fastz(args, ws, rank, local):
         e2e_t.append(time.perf_counter() - t0)
         d2h = res.rec.nbytes + len(res.cigar)
     e2e_ms = sum(e2e_t) / len(e2e_t) * 1e3
-
-    # genome-pair wall time: ASCII sequences + seeds on the host -> alignments + CIGARs on the host
-    # (context creation with device packing, extension, copy-back), seed finding excluded; the context's
-    # teardown (freeing its device memory) happens after the results are on the host and is not counted
-    # device memory of both contexts comes from PyTorch's caching allocator: the benchmark context is closed
-    # first, so the genome-pair context reuses its blocks (a long-running aligner's steady state) instead of
-    # timing cudaMalloc of a fresh ~20 GB traceback pool
     al.close()
-    torch.cuda.synchronize()
-    t0 = time.perf_counter()
-    al2 = fastz.Aligner(w.T, w.Q, device=local, stream=stream.cuda_stream, torch_alloc=True)
-    al2.extend(np.ascontiguousarray(shard))
-    wall_s = time.perf_counter() - t0
-    # NEXT-4 stage on the same pair (rank 0, untimed by the step clock): seeding + ungapped filter
-    seeding = None
-    if rank == 0:
-        try:
-            al2.find_hsps()
-            ts = []
-            for _ in range(3):
-                torch.cuda.synchronize()
-                t1 = time.perf_counter()
-                hs, _an, hits = al2.find_hsps()
-                torch.cuda.synchronize()
-                ts.append(time.perf_counter() - t1)
-            seeding = {"stage": "seeding + ungapped filter (fastz_find_hsps: 12of19 spaced seeds + transitions, "
-                                "x-drop 910, HSP >= 3000), whole pair", "ms": min(ts) * 1e3, "hits": hits,
-                       "hsps": int(len(hs)), "query_mbp_per_s": len(w.Q) / min(ts) / 1e6}
-        except Exception as e:  # reported, never fatal for the headline line
-            seeding = {"error": str(e)[:200]}
-    # NEXT-3 post-pass on the same batch (rank 0, untimed by the step clock): redundant-alignment marking
-    dedup = None
-    if rank == 0:
-        try:
-            al2.mark_redundant()
-            ts = []
-            for _ in range(3):
-                ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                torch.cuda.synchronize()
-                ev0.record(stream)
-                _red, nred = al2.mark_redundant()
-                ev1.record(stream)
-                ev1.synchronize()
-                ts.append(ev0.elapsed_time(ev1))
-            nk = int((al2.results().rec["flags"] & fastz.FLAG_ABOVE_K != 0).sum())
-            dedup = {"stage": "redundant-alignment post-pass (fastz_mark_redundant, reading R14), whole batch, "
-                              "incl. the D2H of the per-seed marks", "ms": min(ts), "above_k": nk,
-                     "redundant": int(nred)}
-        except Exception as e:
-            dedup = {"error": str(e)[:200]}
-    al2.close()
+
+    # secondary: the same device-timed step on C2 (10 Mbp pair, 2^20 seeds per GPU), plus the NEXT-4 seeding
+    # and NEXT-3 post-pass stages on that pair (rank 0)
+    secondary, seeding, dedup = None, None, None
+    if not args.no_secondary:
+        w2, shard2, desc2 = workload(2, 0, ws, rank)
+        al2 = fastz.Aligner(w2.T, w2.Q, device=local, stream=stream.cuda_stream, torch_alloc=True)
+        s2 = torch.from_numpy(np.ascontiguousarray(shard2)).to(dev)
+        al2.extend_only(s2)
+        cells2 = int(al2.census().sum())
+        t2, st2, _l2, _c = measure(al2, s2, 3, 3, stream, flush, ws)
+        ms2 = sum(t2) / len(t2)
+        secondary = {"workload": desc2, "value": cells2 / (ms2 * 1e-3) / 1e9, "unit": "GCUPS", "ms_per_step": ms2,
+                     "inspector_ms": sum(s["ms_inspect"] for s in st2) / len(st2), "cells_per_gpu": cells2,
+                     "roofline_frac": OPS_PER_CELL * cells2 / (sum(s["ms_inspect"] for s in st2) / len(st2) * 1e-3)
+                     / peak_ops}
+        if rank == 0:
+            try:
+                al2.find_hsps()
+                ts = []
+                for _ in range(3):
+                    torch.cuda.synchronize()
+                    t1 = time.perf_counter()
+                    hs, _an, hits = al2.find_hsps()
+                    torch.cuda.synchronize()
+                    ts.append(time.perf_counter() - t1)
+                seeding = {"stage": "seeding + ungapped filter (fastz_find_hsps: 12of19 spaced seeds + transitions, "
+                                    "x-drop 910, HSP >= 3000), C2 pair", "ms": min(ts) * 1e3, "hits": hits,
+                           "hsps": int(len(hs)), "query_mbp_per_s": len(w2.Q) / min(ts) / 1e6}
+            except Exception as e:  # reported, never fatal for the headline line
+                seeding = {"error": str(e)[:200]}
+            try:
+                al2.extend_only(s2)
+                al2.mark_redundant()
+                ts = []
+                for _ in range(3):
+                    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    torch.cuda.synchronize()
+                    ev0.record(stream)
+                    _red, nred = al2.mark_redundant()
+                    ev1.record(stream)
+                    ev1.synchronize()
+                    ts.append(ev0.elapsed_time(ev1))
+                nk = int((al2.results().rec["flags"] & fastz.FLAG_ABOVE_K != 0).sum())
+                dedup = {"stage": "redundant-alignment post-pass (fastz_mark_redundant, reading R14), C2 batch, "
+                                  "incl. the D2H of the per-seed marks", "ms": min(ts), "above_k": nk,
+                         "redundant": int(nred)}
+            except Exception as e:
+                dedup = {"error": str(e)[:200]}
+        al2.close()
+        del w2
 
     t = torch.tensor([ms, e2e_ms, float(cells), float(n)], dtype=torch.float64, device=dev)
     if ws > 1:
@@ -305,16 +411,27 @@ def run_fastz(args, ws, rank, local):
         cells_all, n_all = float(tsum[2]), float(tsum[3])
     else:
         cells_all, n_all = float(cells), float(n)
+    del al
+    gp = None
+    if not args.no_genome_pair:
+        try:
+            gp = genome_pair(ws, rank, local)
+        except Exception as e:  # reported, never fatal for the headline line
+            gp = {"error": str(e)[:300]} if rank == 0 else None
     if rank != 0:
         return
     value = cells_all / (ms * 1e-3) / 1e9
-    insp_ms = sum(insp) / len(insp)
+    insp_ms = sum(s["ms_inspect"] for s in stages) / len(stages)
     achieved = OPS_PER_CELL * cells / (insp_ms * 1e-3)
-    traffic = None
+    traffic, traffic_src = None, None
     tf = os.path.join(ROOT, "profiles", "inspector_traffic.json")
     if os.path.exists(tf):
         try:
-            traffic = json.load(open(tf)).get("bytes_per_launch")
+            tj = json.load(open(tf))
+            entry = tj.get(f"C{args.config}")
+            if entry:
+                traffic = entry.get("bytes_per_launch")
+                traffic_src = "constant from an ncu --set full capture, not measured in this run: " + entry.get("source", "")
         except Exception:
             traffic = None
     avg = lambda k: sum(s[k] for s in stages) / len(stages)  # noqa: E731
@@ -323,28 +440,38 @@ def run_fastz(args, ws, rank, local):
         "ms_per_step": ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
         "data": "synthetic",
         "config": {"workload": desc, "seeds_per_gpu": n, "target_bp": len(w.T), "query_bp": len(w.Q),
-                   "l2": "flushed between timed steps (256 MiB write, untimed)", "rows_per_lane": stages[0].get("R", None)
-                   or int(os.environ.get("FASTZ_R", "4")), "parallelism": f"seed-sharded x{ws}"},
+                   "l2": "flushed between timed steps (256 MiB write, untimed)",
+                   "rows_per_lane": int(os.environ.get("FASTZ_R", "4")), "parallelism": f"seed-sharded x{ws}"},
+    }
+    line.update({
         "seed_extensions_per_s": n_all / (ms * 1e-3),
         "cells": cells_all,
         "clocks": clocks,
         "e2e": {"value": cells_all / (e2e_ms * 1e-3) / 1e9, "unit": "GCUPS", "ms_per_step": e2e_ms,
                 "h2d_bytes_per_step": int(n * 16), "d2h_bytes_per_step": int(d2h)},
         "gpu_launches": launches,
-        "genome_pair_wall_s": wall_s,
+        "genome_pair": gp,
+        "secondary": secondary,
         "seeding": seeding,
         "dedup": dedup,
         "roofline": {"bound": "alu", "kernel": "k_inspect", "achieved": achieved / 1e12, "peak": peak_ops / 1e12,
                      "unit": "Tops/s (INT32 lane ops)", "frac": achieved / peak_ops, "traffic": traffic,
-                     "ops_per_cell": OPS_PER_CELL, "inspector_ms": insp_ms,
-                     "peak_source": f"measured fastz_int_peak (IMNMX/IADD3/VIADDMNMX chains) at {peak_mhz:.0f} MHz"},
+                     "traffic_source": traffic_src, "ops_per_cell": OPS_PER_CELL,
+                     "frac_with_ydrop": OPS_PER_CELL_YDROP * cells / (insp_ms * 1e-3) / peak_ops,
+                     "inspector_ms": insp_ms, "inspector_share_of_step": insp_ms / ms,
+                     "algorithmic": f"{OPS_PER_CELL} int ops per explored cell (P:63, P:346: 4 max + 5 add) x "
+                                    f"{cells} explored cells per launch / mean k_inspect time (CUDA events)",
+                     "peak_source": f"measured fastz_int_peak (IMNMX/IADD3/VIADDMNMX chains on the ALU + FMA pipes, "
+                                    f"128 lane-ops/clk/SM) at {peak_mhz:.0f} MHz; guide-derived 148 SMs x 4 SMSPs x "
+                                    f"2 pipes x 16 lanes/clk x 1.965 GHz = 37.2 T/s"},
         "stages_ms": {k: avg(k) for k in ("ms_upload", "ms_inspect", "ms_bin", "ms_execute", "ms_traceback",
                                           "ms_combine")},
         "bins_per_side": st0["bin_counts"][:7], "exec_sides": st0["n_exec_sides"], "eager_sides": st0["n_eager_sides"],
-        "escalated_sides": st0["n_escalated"], "executor_waves": st0["n_waves"],
-    }
+        "exec_words": st0["exec_words"], "exec_reserved_words": st0["exec_reserved_words"],
+        "wide_sides": st0["n_wide_sides"], "executor_waves": st0["n_waves"],
+    })
     if not args.no_cpu_baseline:
-        line["cpu_baseline"] = cpu_baseline(w, shard)
+        line["cpu_baseline"] = cpu_baseline(w, shard, value / ws)
     print(json.dumps(line), flush=True)
 
 
@@ -357,16 +484,13 @@ def main():
         if args.impl == "reference":
             if rank != 0:
                 return
-            ws_eff = ws
-            run_reference(args, ws_eff, 0)
+            run_reference(args, ws, 0)
             return
         torch.cuda.set_device(local)
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     if args.impl == "reference":
         run_reference(args, ws, rank)
         return
-    if args.profile:
-        args.warmup, args.steps = 1, 1
     run_fastz(args, ws, rank, local)
     if ws > 1:
         import torch.distributed as dist

@@ -25,15 +25,18 @@ def _stale() -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not _stale():
-        return LIB
-    cmd = [NVCC] + FLAGS + ["-o", LIB + ".tmp"] + [os.path.join(CSRC, s) for s in SOURCES]
+def build(force: bool = False, verbose: bool = False, out: str | None = None, defines=()) -> str:
+    """Compile libfastz.so in-tree (``out``/``defines``: an A/B variant of the same sources, e.g.
+    ``-DEXECUTE_MIN_BLOCKS=5`` into ab_libs/, loaded with FASTZ_LIB=...)."""
+    lib = out or LIB
+    if not force and out is None and not _stale():
+        return lib
+    cmd = [NVCC] + FLAGS + list(defines) + ["-o", lib + ".tmp"] + [os.path.join(CSRC, s) for s in SOURCES]
     if verbose:
         print(" ".join(cmd), file=sys.stderr)
     subprocess.check_call(cmd, cwd=CSRC)
-    os.replace(LIB + ".tmp", LIB)
-    return LIB
+    os.replace(lib + ".tmp", lib)
+    return lib
 
 
 if __name__ == "__main__":

@@ -56,7 +56,7 @@ struct fastz_ctx {
     bool t_has_n = false, q_has_n = false;
     DBuf seeds, score, ti, qj, flags, eops, bound, maxsw, esc, nstrip;
     DBuf woff, soff, roff, bin, list, counters, totals, tmpa, tmpb, tmpc, scan_tmp, wl, wlo;
-    DBuf codes, stab, runs, nruns, ciglen, cigar, recs, cells, ring, small, wide, ring2;
+    DBuf codes, stab, runs, nruns, ciglen, cigar, recs, cells, ring, small, wide, ring2, lpt_tmp;
     // seeding (fastz_find_hsps)
     DBuf s_kin, s_kout, s_pin, s_pout, s_start, s_cnt, s_off, s_hits, s_hsp, s_keep, s_sel, s_list, s_list2,
         s_k1, s_k2, s_i1, s_i2, s_flag, s_pos, s_out, s_anch, s_tmp;
@@ -301,7 +301,7 @@ void fastz_destroy(fastz_ctx* c) {
                     &c->flags, &c->eops, &c->bound, &c->maxsw, &c->esc, &c->nstrip, &c->woff, &c->soff, &c->roff, &c->bin, &c->list,
                     &c->counters, &c->totals, &c->tmpa, &c->tmpb, &c->tmpc, &c->scan_tmp, &c->wl, &c->wlo, &c->codes,
                     &c->stab, &c->runs, &c->nruns, &c->ciglen, &c->cigar, &c->recs, &c->cells, &c->ring,
-                    &c->wide, &c->ring2,
+                    &c->wide, &c->ring2, &c->lpt_tmp,
                     &c->small, &c->s_kin, &c->s_kout, &c->s_pin, &c->s_pout, &c->s_start, &c->s_cnt, &c->s_off,
                     &c->s_hits, &c->s_hsp, &c->s_keep, &c->s_sel, &c->s_list, &c->s_list2, &c->s_k1, &c->s_k2,
                     &c->s_i1, &c->s_i2, &c->s_flag, &c->s_pos, &c->s_out, &c->s_anch, &c->s_tmp,
@@ -560,6 +560,7 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
         CK(cudaMemcpyAsync(c->seeds.p, seeds, (size_t)n * 16,
                            seeds_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, st));
     CK(cudaMemsetAsync(c->counters.p, 0, 64 * 4, st));
+    CK(cudaMemsetAsync(c->totals.p, 0, 8 * 8, st));
     long long init = LLONG_MAX;
     CK(cudaMemcpyAsync(c->small.p, &init, sizeof(init), cudaMemcpyHostToDevice, st));
     Batch b = make_batch(c);
@@ -570,8 +571,33 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     ExecPlan pl = make_plan(c);
     const int esc = (c->dp.options & OPT_NO_BLOCK) ? 0 : escalate_strips();
     c->nwide = 0;
+    // experiment (FASTZ_L2_PERSIST=1): keep the boundary rings in a persisting L2 window during the inspector
+    const bool persist = getenv("FASTZ_L2_PERSIST") != nullptr;
+    if (persist) {
+        int maxp = 0, maxw = 0;
+        cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, c->device);
+        cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, c->device);
+        const size_t ringb = (size_t)c->nslots * (size_t)(c->rmask + 1) * sizeof(int4);
+        cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, std::min<size_t>((size_t)maxp, ringb));
+        cudaStreamAttrValue a{};
+        a.accessPolicyWindow.base_ptr = c->ring.p;
+        a.accessPolicyWindow.num_bytes = std::min<size_t>(ringb, (size_t)maxw);
+        a.accessPolicyWindow.hitRatio = std::min(1.0f, (float)maxp / (float)a.accessPolicyWindow.num_bytes);
+        a.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        a.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &a);
+        if (getenv("FASTZ_VERBOSE"))
+            fprintf(stderr, "L2 persist: max set-aside %d B, max window %d B, ring %zu B, hitRatio %.3f\n", maxp, maxw,
+                    ringb, a.accessPolicyWindow.hitRatio);
+    }
     CK(launch_inspect(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, esc > 0 ? esc : INT_MAX,
                       nullptr, 0, st));
+    if (persist) {
+        cudaStreamAttrValue a{};
+        a.accessPolicyWindow.num_bytes = 0;
+        cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &a);
+        cudaCtxResetPersistingL2Cache();
+    }
     if (esc > 0) CK(launch_inspect_block(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, st));
     CK(cudaEventRecord(c->ev[2], st));
     CK(launch_bin(c->R, c->dp, sa, (int)ns, pl, c->scan_tmp.p, stb, P_<long long>(c->tmpa), P_<long long>(c->tmpb),
@@ -640,6 +666,13 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     const long long words = h.totals[0], strips = h.totals[1], nrun = h.totals[2];
     c->nexec = h.totals[3];
     const long long nblock = h.totals[4];
+    if (nblock > 1) {  // LPT inside the block-per-side bins; the total words are unchanged
+        const size_t lb = lpt_tmp_bytes((int)nblock);
+        AL(lpt_tmp, lb);
+        CK(launch_lpt(pl, (int)nblock, (int)c->nexec, P_<long long>(c->tmpa), P_<long long>(c->wl),
+                      P_<long long>(c->wlo), P_<int>(c->tmpb), c->lpt_tmp.p, c->lpt_tmp.cap, c->scan_tmp.p, stb, st));
+        extra_launches += 3;
+    }
     AL(stab, std::max<long long>(strips, 1) * 8);
     AL(runs, std::max<long long>(nrun, 1) * 4);
     // traceback-code pool: one wave if it fits the budget, else consecutive ranges of the executor list
@@ -654,7 +687,8 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
         } else {
             size_t fr = 0, tot = 0;  // cudaMemGetInfo costs milliseconds: only when the pool must grow
             cudaMemGetInfo(&fr, &tot);
-            budget_words = (long long)((fr + c->codes.cap) / 2 / 4);
+            // 80% of what is free (plus the pool itself): waves cost a tail each, so use the memory
+            budget_words = (long long)((double)(fr + c->codes.cap) * 0.8 / 4);
         }
     }
     std::vector<std::pair<long long, long long>> waves;  // list ranges [a, b)
@@ -710,8 +744,16 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     long long* dtotal = P_<long long>(c->small) + 1;
     CK(launch_combine_len(c->dp, b, sa, pl, o, c->scan_tmp.p, stb, dtotal, st));
     long long ctot = 0;
+    int nfail = 0;
+    long long h_written = 0;
     CK(cudaMemcpyAsync(&ctot, dtotal, sizeof(ctot), cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));  // host sync 2: CIGAR bytes
+    CK(cudaMemcpyAsync(&h_written, P_<long long>(c->totals) + 6, sizeof(h_written), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(&nfail, P_<int>(c->counters) + 26, sizeof(nfail), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));  // host sync 2: CIGAR bytes, executor self-check
+    if (nfail)
+        return fail(FASTZ_ECUDA, "executor self-check failed on " + std::to_string(nfail) +
+                                     " sides (S(i*,j*) differs from the inspector's peak, or a traceback-code store "
+                                     "left the side's reservation)");
     AL(cigar, std::max<long long>(ctot, 1));
     o = make_out(c);
     CK(launch_combine_write(c->dp, b, sa, pl, o, st));
@@ -726,7 +768,8 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     S.n_exec_sides = c->nexec;
     S.n_eager_sides = h.counters[2];
     for (int k = 0; k < 7; ++k) S.bin_counts[k] = h.counters[2 + k];
-    S.exec_words = words;
+    S.exec_words = h_written;
+    S.exec_reserved_words = words;
     S.cigar_bytes = ctot;
     S.n_waves = c->nwaves;
     S.n_escalated = h.counters[21];

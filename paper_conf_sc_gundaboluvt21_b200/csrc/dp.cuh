@@ -52,6 +52,7 @@ constexpr int SUBTAB_INTS = SubTab<true>::INTS;  // shared allocation (the large
 // side flags
 constexpr uint32_t SF_EAGER = 1u, SF_OVERFLOW = 2u, SF_RING = 4u, SF_ESCALATE = 8u, SF_NOTB = 16u;
 constexpr uint32_t SF_WIDE = 32u;  // inspected with the wide ring (band wider than the regular ring)
+constexpr uint32_t SF_CHECKFAIL = 64u;  // executor self-check failed (S(i*, j*) mismatch or a store past the reservation)
 constexpr int OPT_NO_EAGER = 1, OPT_NO_TRIM = 2, OPT_NO_BINNING = 4, OPT_NO_BLOCK = 8, OPT_TB_ABOVE_K = 16;
 
 struct DevParams {

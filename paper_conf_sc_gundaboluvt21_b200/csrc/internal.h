@@ -78,6 +78,11 @@ cudaError_t launch_bin(int R, const DevParams& P, const SideArrays& sa, int nsid
                        size_t scan_tmp_bytes, long long* tmp_a, long long* tmp_b, long long* tmp_c,
                        cudaStream_t st);
 size_t scan_tmp_bytes(int n);
+// LPT order of the block-per-side executor sides list[0, nblock) (descending words), offsets recomputed
+size_t lpt_tmp_bytes(int n);
+cudaError_t launch_lpt(const ExecPlan& pl, int nblock, int nexec, const long long* words, long long* keys_in,
+                       long long* keys_out, int* vals_in, void* sort_tmp, size_t sort_tmp_bytes, void* scan_tmp,
+                       size_t scan_tmp_bytes, cudaStream_t st);
 // list the sides flagged SF_WIDE (any order) and count them
 cudaError_t launch_wide_list(const SideArrays& sa, int nsides, int* list, int* count, cudaStream_t st);
 // redundant-alignment post-pass (dedup.cu; NEXT-3, reading R14)

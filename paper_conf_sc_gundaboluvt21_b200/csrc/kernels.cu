@@ -1,5 +1,6 @@
 // kernels.cu -- sm_100a kernels of the FastZ hot path: pack, inspector, census, binning, executor,
 // traceback, CIGAR assembly.  Citations P:<n> are PAPER.md lines; readings R1..R8 are in DESIGN.md.
+#include <cub/device/device_radix_sort.cuh>
 #include <cub/device/device_scan.cuh>
 
 #include "../../include/fastz.h"
@@ -169,6 +170,9 @@ __device__ __forceinline__ void io_init(SideIO& io, SmemDP& sm, int4* ring, int 
     io.wi = warp;
     io.K = WARPS;
     io.maxsw = 0;
+    io.wlim = 0;
+    io.xexp = 0;
+    io.written = nullptr;
 }
 
 // eager traceback by lane 0 over the 17x17 corner codes; returns ops (2 bits each, peak -> origin)
@@ -343,11 +347,12 @@ __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int
 // Trimmed executor: the DP over [0,i*]x[0,j*] only, writing traceback codes.  Length binning
 // as a schedule: the CTAs first take the long sides (bins >= 3, block per side, strips pipelined
 // across the CTA's warps), then every warp takes short sides (bins 1-2, warp per side), larger bins first.
-#ifdef EXECUTE_MIN_BLOCKS
-#define EXECUTE_ATTR __launch_bounds__(WARPS * 32, EXECUTE_MIN_BLOCKS)
-#else
-#define EXECUTE_ATTR __launch_bounds__(WARPS * 32)
+// 6 resident CTAs per SM (<= 80 registers): the per-step instruction count of the warp-per-side loop is the same
+// as at its natural 96 registers (5 CTAs), so the extra occupancy is free (SASS: 95 vs 94.5 per 4-cell step)
+#ifndef EXECUTE_MIN_BLOCKS
+#define EXECUTE_MIN_BLOCKS 6
 #endif
+#define EXECUTE_ATTR __launch_bounds__(WARPS * 32, EXECUTE_MIN_BLOCKS)
 template <int R, bool NM>
 __global__ void EXECUTE_ATTR k_execute(DevParams P, Batch b, int4* ring, int rmask,
                                                          SideArrays sa, ExecPlan pl, int lo, int hi, int nblock,
@@ -382,9 +387,12 @@ __global__ void EXECUTE_ATTR k_execute(DevParams P, Batch b, int4* ring, int rma
         io.codes = out.codes + (pl.woff[side] - base);
         io.stab = out.stab + pl.soff[side];
         io.maxsw = sa.maxsw[side];
+        io.xexp = (P.options & OPT_NO_TRIM) ? INT_MIN : sa.score[side] - P.OE;
+        io.written = (unsigned long long*)(pl.totals + 6);
         SideOut o;
         run_side<R, MODE_EXEC, false, true, NM>(P, io, o);
         if (threadIdx.x == 0 && (o.flags & SF_RING)) atomicOr(&sa.flags[side], SF_RING);
+        if (threadIdx.x == 0 && o.checkfail) atomicAdd(&pl.counters[26], 1);
         __syncthreads();
     }
     SideIO io;
@@ -403,9 +411,13 @@ __global__ void EXECUTE_ATTR k_execute(DevParams P, Batch b, int4* ring, int rma
         }
         io.codes = out.codes + (pl.woff[side] - base);
         io.stab = out.stab + pl.soff[side];
+        io.wlim = sa.bound[side];
+        io.xexp = (P.options & OPT_NO_TRIM) ? INT_MIN : sa.score[side] - P.OE;
+        io.written = (unsigned long long*)(pl.totals + 6);
         SideOut o;
         run_side<R, MODE_EXEC, false, false, NM>(P, io, o);
         if (lane == 0 && (o.flags & SF_RING)) atomicOr(&sa.flags[side], SF_RING);
+        if (lane == 0 && o.checkfail) atomicAdd(&pl.counters[26], 1);
         __syncwarp();
     }
 }
@@ -463,8 +475,9 @@ __global__ void k_traceback(SideArrays sa, ExecPlan pl, int lo, int hi, long lon
         }
         const uint32_t code = (w >> ((((t % SPW) * R) + k) * 4)) & 15u;
         // branch-free step (the 32 walks of a warp diverge otherwise): in state S the cell's source decides
-        // (H -> M, D -> enter D, I -> enter I), in a gap state the move is the gap's; one op per iteration
-        const int eff = state == 0 ? (int)(code & 3u) : state;  // 0 M, 1 D, 2 I
+        // (H -> M, D -> enter D, I -> enter I; executor code: bit 1 = I, else bit 0 = D), in a gap state the
+        // move is the gap's; one op per iteration
+        const int eff = state == 0 ? ((code & 2u) ? 2 : (int)(code & 1u)) : state;  // 0 M, 1 D, 2 I
         const uint32_t op = eff == 0 ? (uint32_t)OP_M : (eff == 1 ? (uint32_t)OP_D : (uint32_t)OP_I);
         const bool ext = eff == 1 ? ((code >> 2) & 1u) : ((code >> 3) & 1u);
         state = eff == 0 ? 0 : (ext ? eff : 0);
@@ -536,7 +549,7 @@ __global__ void __launch_bounds__(128) k_traceback_warp(SideArrays sa, ExecPlan 
         }
         const uint32_t w = wbuf[(wr - rlo) * 32 + ln];
         const uint32_t code = (w >> ((((t % SPW) * R) + k) * 4)) & 15u;
-        const int eff = state == 0 ? (int)(code & 3u) : state;  // 0 M, 1 D, 2 I
+        const int eff = state == 0 ? ((code & 2u) ? 2 : (int)(code & 1u)) : state;  // 0 M, 1 D, 2 I
         const uint32_t op = eff == 0 ? (uint32_t)OP_M : (eff == 1 ? (uint32_t)OP_D : (uint32_t)OP_I);
         const bool ext = eff == 1 ? ((code >> 2) & 1u) : ((code >> 3) & 1u);
         state = eff == 0 ? 0 : (ext ? eff : 0);
@@ -639,6 +652,41 @@ cudaError_t launch_wide_list(const SideArrays& sa, int nsides, int* list, int* c
     cudaError_t e = cudaMemsetAsync(count, 0, 4, st);
     if (e != cudaSuccess || nsides == 0) return e;
     k_wide_list<<<(nsides + 255) / 256, 256, 0, st>>>(sa, nsides, list, count);
+    return cudaGetLastError();
+}
+
+// LPT order inside the block-per-side bins (long problems first): list[0, nblock) sorted by descending
+// executor words (proportional to the trimmed cells), then the pool offsets are recomputed in the new list order.
+__global__ void k_lpt_keys(ExecPlan pl, const long long* words, int nblock, long long* keys, int* vals) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < nblock) {
+        const int side = pl.list[i];
+        keys[i] = words[side];
+        vals[i] = side;
+    }
+}
+
+size_t lpt_tmp_bytes(int n) {
+    size_t bytes = 0;
+    cub::DeviceRadixSort::SortPairsDescending(nullptr, bytes, (const long long*)nullptr, (long long*)nullptr,
+                                              (const int*)nullptr, (int*)nullptr, n > 0 ? n : 1);
+    return bytes;
+}
+
+cudaError_t launch_lpt(const ExecPlan& pl, int nblock, int nexec, const long long* words, long long* keys_in,
+                       long long* keys_out, int* vals_in, void* sort_tmp, size_t sort_tmp_bytes, void* scan_tmp,
+                       size_t scan_tmp_bytes, cudaStream_t st) {
+    if (nblock < 2) return cudaSuccess;
+    k_lpt_keys<<<(nblock + 255) / 256, 256, 0, st>>>(pl, words, nblock, keys_in, vals_in);
+    size_t b = sort_tmp_bytes;
+    cudaError_t e = cub::DeviceRadixSort::SortPairsDescending(sort_tmp, b, keys_in, keys_out, vals_in, pl.list, nblock,
+                                                              0, 64, st);
+    if (e != cudaSuccess) return e;
+    const int g = (nexec + 255) / 256;
+    k_list_words<<<g, 256, 0, st>>>(pl, words, pl.wl, nexec);
+    b = scan_tmp_bytes;
+    if ((e = cub::DeviceScan::ExclusiveSum(scan_tmp, b, pl.wl, pl.wlo, nexec, st)) != cudaSuccess) return e;
+    k_list_offsets<<<g, 256, 0, st>>>(pl, pl.wlo, pl.wl);
     return cudaGetLastError();
 }
 

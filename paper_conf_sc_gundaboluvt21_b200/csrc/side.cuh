@@ -99,6 +99,11 @@ struct SideIO {
     PipeShared* ps;                     // PIPE: shared side state
     int wi, K;                          // PIPE: warp index in the CTA, warps per side
     int maxsw;                          // PIPE executor: words reserved per strip (from the inspector)
+    long long wlim;                     // SOLO executor: words reserved for the side (stores beyond are dropped
+                                        // and reported: the executor self-check)
+    int xexp;                           // executor: X (= S - O - E) the inspector found at (M, N) = (i*, j*)
+                                        // (INT_MIN: not checked -- the untrimmed ablation ends elsewhere)
+    unsigned long long* written;        // executor: code words written (all sides; stats)
 };
 
 struct SideOut {
@@ -110,6 +115,7 @@ struct SideOut {
     long long words;         // all strips' words (inspector: the untrimmed executor's storage)
     int maxsw_all;           // widest strip over all strips
     int nstrips;             // strips run
+    int checkfail;           // executor self-check: 1 = S(i*, j*) != inspector score or a store past the reservation
 };
 
 template <int R>
@@ -147,6 +153,14 @@ __device__ __forceinline__ int4 boundary(const int4* __restrict__ ring, int rmas
 
 __device__ __forceinline__ void pipe_wait() { __nanosleep(100); }
 
+// executor traceback code bit: cw += bit if a > b, as one ISETP (ALU pipe) + one predicated IMAD (FMA pipe; `one`
+// is a runtime 1 so ptxas cannot turn it into an ALU-pipe IADD3).  The bits of a word never overlap, so the add
+// is an OR.
+__device__ __forceinline__ void code_bit_gt(uint32_t& cw, int a, int b, uint32_t bit, int one) {
+    asm("{ .reg .pred p; setp.gt.s32 p, %1, %2; @p mad.lo.u32 %0, %3, %4, %0; }"
+        : "+r"(cw) : "r"(a), "r"(b), "r"(bit), "r"(one));
+}
+
 template <int R, int MODE, bool EAGER, bool PIPE, bool NM>
 __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, SideOut& out) {
     constexpr int H = StripGeom<R>::H;
@@ -178,6 +192,8 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
     int maxsw = 0, bound_maxsw = 0, nstr = 0;
     uint32_t flags = 0;
     bool upd = false;
+    bool bad = false;        // executor self-check
+    int xcap = INT_MIN;      // executor: X at (M, N)
 
     for (int s = PIPE ? io.wi : 0;; s += PIPE ? io.K : 1) {
         const int slot = s % PIPE_SLOTS, pslot = (s + PIPE_SLOTS - 1) % PIPE_SLOTS;
@@ -358,7 +374,21 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                     const int h = fma_add(vs[k], one, xd);  // X_diag + sub(a_i, b_j) + O + E
                     const int d = __viaddmax_s32(du, mE, xu);
                     const int iv = __viaddmax_s32(I[k], mE, X[k]);
-                    const int sr = __vimax3_s32(h, d, iv);
+                    int sr;
+                    if constexpr (MODE == MODE_EXEC) {
+                        // traceback code (P:178's 2 + 1 + 1 bits), executor format: bit 0 d > h, bit 1 iv > max(h, d)
+                        // (S source: I if bit 1, else D if bit 0, else H -- reading R4's H > D > I), bit 2 d > xu
+                        // (D extends: strictly better than opening, R4b), bit 3 iv > X_left (I extends)
+                        const int mhd = imax(h, d);
+                        sr = imax(mhd, iv);
+                        const uint32_t sh = (uint32_t)((((j % SPW) * R) + k) * 4);
+                        code_bit_gt(cw, d, h, 1u << sh, one);
+                        code_bit_gt(cw, iv, mhd, 2u << sh, one);
+                        code_bit_gt(cw, d, xu, 4u << sh, one);
+                        code_bit_gt(cw, iv, X[k], 8u << sh, one);
+                    } else {
+                        sr = __vimax3_s32(h, d, iv);
+                    }
                     // live iff S_raw >= thr = max(W_up, W_left) (reading R3); W = max(thr, S_raw - Y) equals
                     // max(thr, S_live - Y) because a dead cell has S_raw - Y < S_raw < thr.  thr comes from the
                     // row above and the previous column (ready before S), so the dependent chain after S is one
@@ -367,10 +397,6 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
                     const int thr = imax(wu, W[k]);
                     const int xn = kill_fma(sr, thr, mOE, one, zero);
                     const int wn = __viaddmax_s32(sr, mY, thr);
-                    if constexpr (MODE == MODE_EXEC) {
-                        const uint32_t code = cell_code(h, d, iv, du, xu, I[k], X[k], E);
-                        cw |= code << ((((j % SPW) * R) + k) * 4);
-                    }
                     if constexpr (EG) {
                         const int r = r0 + k, c = start + rc;
                         if (r <= io.eager_max && c <= io.eager_max)
@@ -434,7 +460,10 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             st_shared4_if(is31, sgo + 16u * (unsigned)j, bq);
             if constexpr (MODE == MODE_EXEC) {
                 if ((j % SPW) == SPW - 1) {  // j == tt mod 4 and SPW divides 4
-                    io.codes[wbase + (long long)(tt / SPW) * 32 + lane] = cw;
+                    const long long wl = (long long)(tt / SPW) * 32 + lane;
+                    // never past the reservation (PIPE: the strip's stride, SOLO: the side's words)
+                    if (PIPE ? wl < io.maxsw : wbase + wl < io.wlim) io.codes[wbase + wl] = cw;
+                    else bad = true;
                     cw = 0;
                 }
             }
@@ -535,7 +564,11 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         __syncwarp();
         park(t, tfinal);  // the last (partial) block's bottom rows
         if constexpr (MODE == MODE_EXEC) {
-            if ((tfinal % SPW) != SPW - 1) io.codes[wbase + (long long)(tfinal / SPW) * 32 + lane] = cw;
+            if ((tfinal % SPW) != SPW - 1) {
+                const long long wl = (long long)(tfinal / SPW) * 32 + lane;
+                if (PIPE ? wl < io.maxsw : wbase + wl < io.wlim) io.codes[wbase + wl] = cw;
+                else bad = true;
+            }
         }
         const int Wtail = ws->bout[tfinal & (BK - 1)].z;
         const int sw = (tfinal / SPW + 1) * 32;
@@ -554,11 +587,35 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             bound_maxsw = ps->bound_maxsw;
             flags = ps->flags;
         }
+        if constexpr (MODE == MODE_INSPECT && !PIPE) {
+        }
+        if constexpr (MODE == MODE_EXEC) {
+            // self-check input: the lane holding row M ends the strip with X(M, N) in its registers (the peak
+            // (M, N) = (i*, j*) is live, so the strip cannot have stopped before that lane reached column N)
+#pragma unroll
+            for (int k = 0; k < R; ++k)
+                if (r0 + k == M) xcap = X[k];
+            if (__any_sync(FULL, bad)) flags |= SF_CHECKFAIL;
+            if (lane == 0) atomicAdd(io.written, (unsigned long long)sw);
+        }
+        const int maxsw_prev = maxsw;
         cum_words += sw;
         maxsw = sw > maxsw ? sw : maxsw;
         if (MODE == MODE_INSPECT && anyupd) {
-            bound_words = cum_words;
-            bound_maxsw = maxsw;
+            // Storage of the trimmed executor, sized from the inspector ("allocate ... according to the
+            // exact size needed"): the executor runs strips 0..s* = i*/H and its strip k covers columns
+            // [start_k, j*] only, stopping no later than this strip did, i.e. min(tfinal, j* - start + 31) steps.
+            // The bound is taken whenever a lane's peak moves: full widths for the strips above, the trimmed
+            // width of this strip (with the warp's largest peak column, an upper bound of j*); exact for peaks in
+            // the last strip with an update, an upper bound otherwise.
+            int mbj = bj == INT_MAX ? 0 : bj;
+#pragma unroll
+            for (int off = 16; off; off >>= 1) mbj = imax(mbj, __shfl_xor_sync(FULL, mbj, off));
+            const int sp = mbj - start > 0 ? mbj - start : 0;
+            const int tt2 = tfinal < sp + 31 ? tfinal : sp + 31;
+            const int tw = (tt2 / SPW + 1) * 32;
+            bound_words = cum_words - sw + tw;
+            bound_maxsw = imax(maxsw_prev, tw);
         }
         bool over = false;
         if (e - start + 4 > rmask) {  // strip wider than the ring: the parked row has been overwritten
@@ -613,6 +670,11 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
         }
     }
 side_done:
+    if constexpr (MODE == MODE_EXEC) {  // X at (i*, j*) -> best (the PIPE block below takes the max over warps)
+        best = xcap;
+#pragma unroll
+        for (int off = 16; off; off >>= 1) best = imax(best, __shfl_xor_sync(FULL, best, off));
+    }
     if constexpr (MODE == MODE_INSPECT) {
 #pragma unroll
         for (int off = 16; off; off >>= 1) {
@@ -665,6 +727,8 @@ side_done:
     out.words = cum_words;
     out.maxsw_all = maxsw;
     out.nstrips = nstr;
+    // executor self-check: the recomputed S(i*, j*) equals the inspector's peak, no store left the reservation
+    out.checkfail = (MODE == MODE_EXEC && ((flags & SF_CHECKFAIL) || (io.xexp != INT_MIN && best != io.xexp))) ? 1 : 0;
 }
 
 // Reset the block-per-problem shared state before a side (one thread; caller synchronises the CTA).

@@ -6,7 +6,8 @@ collectives sit at the edges of the path:
 1. rank ``src`` packs the two sequences to 2 bits per base on its GPU (``fastz_pack_sequence``) and broadcasts
    the packed words (+ N masks when present) and the seed list over NCCL; every rank builds its context from
    the packed device buffers (``fastz_create_packed``: reversed copies made on its own GPU);
-2. seeds are permuted by a fixed hash and cut into W contiguous shards (spreads the unknown-length long tail);
+2. seeds are permuted by a fixed low-discrepancy stride and cut into W contiguous shards (spreads the
+   unknown-length long tail);
 3. every rank runs the CUDA path on its shard (no communication);
 4. per-rank record counts / CIGAR sizes are all-gathered, the device-resident records (64 B each) and CIGAR
    bytes are gathered to ``src`` over NCCL, and ``src`` restores seed order with index arithmetic on its GPU
@@ -25,24 +26,35 @@ import torch.distributed as dist
 
 from . import fastz
 
-_HASH = np.uint64(0x9E3779B97F4A7C15)
 REC_BYTES = 64  # fastz_alignment
 _OFF_I64 = 6    # cigar_off: int64 word 6 of a record (byte 48)
 _LEN_I32 = 14   # cigar_len: int32 word 14 of a record (byte 56)
 
 
+def _stride(n: int) -> int:
+    """An odd multiplier near n / golden ratio, coprime with n: k -> k * a mod n is a bijection of [0, n)."""
+    import math
+    a = max(1, int(n * 0.6180339887498949)) | 1
+    while math.gcd(a, n) != 1:
+        a += 2
+    return a
+
+
 def shard_order(n: int) -> np.ndarray:
-    """Deterministic pseudo-random permutation of seed indices (multiplicative hash, stable argsort)."""
-    h = (np.arange(n, dtype=np.uint64) * _HASH) ^ np.uint64(0xD1B54A32D192ED03)
-    h ^= h >> np.uint64(29)
-    return np.argsort(h, kind="stable").astype(np.int64)
+    """Deterministic low-discrepancy permutation of seed indices (position k holds seed k * a mod n): each
+    rank's contiguous range of it samples the whole seed list evenly, so the unknown-length long tail spreads."""
+    if n == 0:
+        return np.zeros(0, dtype=np.int64)
+    return (np.arange(n, dtype=np.int64) * _stride(n)) % n
 
 
 def shard_indices(n: int, world: int, rank: int) -> np.ndarray:
-    order = shard_order(n)
+    """Seed indices of ``rank``'s shard (sorted): positions [n*rank/W, n*(rank+1)/W) of shard_order(n)."""
     lo = (n * rank) // world
     hi = (n * (rank + 1)) // world
-    return np.sort(order[lo:hi])
+    if hi <= lo:
+        return np.zeros(0, dtype=np.int64)
+    return np.sort((np.arange(lo, hi, dtype=np.int64) * _stride(n)) % n)
 
 
 def _world(group=None):
@@ -177,14 +189,16 @@ def _broadcast_packed(seq, src: int, group, device: int, stream) -> fastz.Packed
 
 
 def extend_genome_pair(T: bytes | None, Q: bytes | None, seeds: np.ndarray | None, params=None, group=None,
-                       extend_fn=None, src: int = 0, mark_redundant: bool = False, mark_fn=None, timings=None):
+                       extend_fn=None, src: int = 0, mark_redundant: bool = False, mark_fn=None, timings=None,
+                       torch_alloc: bool = False):
     """Collective: every rank calls it; only ``src`` needs real inputs.  Returns (records, cigar) on ``src`` as
     host arrays (ALIGN_DTYPE, bytes) in seed order, (None, None) elsewhere.
 
     ``mark_redundant``: after the gather, ``src`` runs the redundant-alignment post-pass (NEXT-3, reading R14)
     over the WHOLE record set -- the marks depend on every record, so they cannot be taken per shard -- setting
     FLAG_REDUNDANT (``mark_fn(rec)`` on host records if given, else the CUDA post-pass on the device records).
-    ``timings``: optional dict that receives per-phase seconds on this rank."""
+    ``timings``: optional dict that receives per-phase seconds on this rank.  ``torch_alloc``: the context's
+    device memory comes from PyTorch's caching allocator (a long-running driver reuses it across pairs)."""
     import time
     world, rank = _world(group)
     dev = _dev(group)
@@ -211,7 +225,7 @@ def extend_genome_pair(T: bytes | None, Q: bytes | None, seeds: np.ndarray | Non
     t1 = time.perf_counter()
     # 2. the CUDA path on this rank's shard
     if extend_fn is None:
-        with fastz.Aligner(pT, pQ, params, device=device, stream=stream) as al:
+        with fastz.Aligner(pT, pQ, params, device=device, stream=stream, torch_alloc=torch_alloc) as al:
             al.extend_only(sd[idx])
             rec, cig = al.results_device()
             rec, cig = rec.clone(), cig.clone()  # the context's memory is released on exit

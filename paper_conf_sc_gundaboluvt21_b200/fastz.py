@@ -15,12 +15,14 @@ from dataclasses import dataclass, field
 import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libfastz.so")
+# FASTZ_LIB: an alternative build of the same library (A/B experiments, tools/); default the in-tree build
+LIB_PATH = os.environ.get("FASTZ_LIB") or os.path.join(HERE, "libfastz.so")
 
 FASTZ_OK, FASTZ_EINVAL, FASTZ_EBASE, FASTZ_ERANGE = 0, -1, -2, -3
 FASTZ_ENOMEM, FASTZ_ECUDA, FASTZ_ETRUNC, FASTZ_ESTATE = -4, -5, -6, -7
 FLAG_ABOVE_K, FLAG_LEFT_EAGER, FLAG_RIGHT_EAGER, FLAG_OVERFLOW, FLAG_NO_CIGAR, FLAG_REDUNDANT = 1, 2, 4, 8, 16, 32
 OPT_NO_EAGER, OPT_NO_TRIM, OPT_NO_BINNING, OPT_NO_BLOCK, OPT_TRACEBACK_ABOVE_K = 1, 2, 4, 8, 16
+OPT_QUERY_REVCOMP = 32
 
 # names declared in include/fastz.h (checked by tests/test_abi.py against the header)
 EXPORTS = ["fastz_default_params", "fastz_create", "fastz_extend_seeds", "fastz_get_alignments",
@@ -147,8 +149,8 @@ def _ptr_len(x):
     if isinstance(x, str):
         x = x.encode()
     if isinstance(x, (bytes, bytearray)):
-        buf = ctypes.create_string_buffer(bytes(x), len(x))
-        return ctypes.addressof(buf), len(x), False, buf
+        arr = np.frombuffer(x, dtype=np.uint8)  # zero-copy view (the library only reads host inputs)
+        return (arr.ctypes.data if len(x) else None), len(x), False, (arr, x)
     arr = np.ascontiguousarray(x)
     return arr.ctypes.data, arr.nbytes, False, arr
 
@@ -218,7 +220,7 @@ class _DevView:
     """__cuda_array_interface__ over library-owned device memory (zero-copy torch.as_tensor)."""
 
     def __init__(self, ptr: int, nbytes: int):
-        self.__cuda_array_interface__ = {"shape": (nbytes,), "typestr": "|u1", "data": (ptr or 0, True),
+        self.__cuda_array_interface__ = {"shape": (nbytes,), "typestr": "|u1", "data": (ptr or 0, False),
                                          "version": 3, "strides": None}
 
 
