@@ -28,7 +28,7 @@ def _stale() -> bool:
 def build(force: bool = False, verbose: bool = False, out: str | None = None, defines=()) -> str:
     """Compile libfastz.so in-tree (``out``/``defines``: an A/B variant of the same sources, e.g.
     ``-DEXECUTE_MIN_BLOCKS=5`` into ab_libs/, loaded with FASTZ_LIB=...)."""
-    lib = out or LIB
+    lib = os.path.abspath(out) if out else LIB
     if not force and out is None and not _stale():
         return lib
     cmd = [NVCC] + FLAGS + list(defines) + ["-o", lib + ".tmp"] + [os.path.join(CSRC, s) for s in SOURCES]

@@ -56,7 +56,7 @@ struct fastz_ctx {
     bool t_has_n = false, q_has_n = false;
     DBuf seeds, score, ti, qj, flags, eops, bound, maxsw, esc, nstrip;
     DBuf woff, soff, roff, bin, list, counters, totals, tmpa, tmpb, tmpc, scan_tmp, wl, wlo;
-    DBuf codes, stab, runs, nruns, ciglen, cigar, recs, cells, ring, small, wide, ring2, lpt_tmp;
+    DBuf codes, stab, runs, nruns, ciglen, cigar, recs, cells, ring, small, wide, ring2, lpt_tmp, order_tmp, order_buf;
     // seeding (fastz_find_hsps)
     DBuf s_kin, s_kout, s_pin, s_pout, s_start, s_cnt, s_off, s_hits, s_hsp, s_keep, s_sel, s_list, s_list2,
         s_k1, s_k2, s_i1, s_i2, s_flag, s_pos, s_out, s_anch, s_tmp;
@@ -301,7 +301,7 @@ void fastz_destroy(fastz_ctx* c) {
                     &c->flags, &c->eops, &c->bound, &c->maxsw, &c->esc, &c->nstrip, &c->woff, &c->soff, &c->roff, &c->bin, &c->list,
                     &c->counters, &c->totals, &c->tmpa, &c->tmpb, &c->tmpc, &c->scan_tmp, &c->wl, &c->wlo, &c->codes,
                     &c->stab, &c->runs, &c->nruns, &c->ciglen, &c->cigar, &c->recs, &c->cells, &c->ring,
-                    &c->wide, &c->ring2, &c->lpt_tmp,
+                    &c->wide, &c->ring2, &c->lpt_tmp, &c->order_tmp, &c->order_buf,
                     &c->small, &c->s_kin, &c->s_kout, &c->s_pin, &c->s_pout, &c->s_start, &c->s_cnt, &c->s_off,
                     &c->s_hits, &c->s_hsp, &c->s_keep, &c->s_sel, &c->s_list, &c->s_list2, &c->s_k1, &c->s_k2,
                     &c->s_i1, &c->s_i2, &c->s_flag, &c->s_pos, &c->s_out, &c->s_anch, &c->s_tmp,
@@ -571,6 +571,8 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     ExecPlan pl = make_plan(c);
     const int esc = (c->dp.options & OPT_NO_BLOCK) ? 0 : escalate_strips();
     c->nwide = 0;
+    if (getenv("FASTZ_TEST_SELFCHECK")) c->dp.options |= OPT_SELFCHECK_TEST;  // tests: the self-check must fire
+    else c->dp.options &= ~OPT_SELFCHECK_TEST;
     // experiment (FASTZ_L2_PERSIST=1): keep the boundary rings in a persisting L2 window during the inspector
     const bool persist = getenv("FASTZ_L2_PERSIST") != nullptr;
     if (persist) {
@@ -590,8 +592,25 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
             fprintf(stderr, "L2 persist: max set-aside %d B, max window %d B, ring %zu B, hitRatio %.3f\n", maxp, maxw,
                     ringb, a.accessPolicyWindow.hitRatio);
     }
+    // inspector order: predicted-longest sides first (FASTZ_INSPECT_ORDER=0: seed order)
+    int* order = nullptr;
+    bool ordered = false;
+    {
+        const char* e = getenv("FASTZ_INSPECT_ORDER");
+        ordered = ns > 1 && !(e && atoi(e) == 0);
+    }
+    if (ordered) {
+        const size_t ob = order_tmp_bytes((int)ns);
+        AL(order_tmp, ob);
+        AL(order_buf, (size_t)ns * 4);
+        // keys in/out in tmpa (2 x u32 per side), values in tmpb (the binning scratch is free until launch_bin)
+        unsigned* kin = reinterpret_cast<unsigned*>(P_<long long>(c->tmpa));
+        CK(launch_order(b, c->dp, (int)ns, kin, kin + ns, P_<int>(c->tmpb), P_<int>(c->order_buf), c->order_tmp.p,
+                        c->order_tmp.cap, st));
+        order = P_<int>(c->order_buf);
+    }
     CK(launch_inspect(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, esc > 0 ? esc : INT_MAX,
-                      nullptr, 0, st));
+                      order, ordered ? (int)ns : 0, st));
     if (persist) {
         cudaStreamAttrValue a{};
         a.accessPolicyWindow.num_bytes = 0;
@@ -647,12 +666,13 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
             CK(cudaMemcpyAsync(wl, c->wide.p, (size_t)nw * 4, cudaMemcpyDeviceToDevice, st));
             CK(cudaMemsetAsync(c->counters.p, 0, 64 * 4, st));
             CK(launch_inspect(c->R, c->grid2, c->dp, b, P_<int4>(c->ring2), c->rmask2, sa, pl, INT_MAX, wl, nw, st));
+            CK(launch_mark_wide(sa, wl, nw, st));
             CK(cudaMemsetAsync(c->counters.p, 0, 64 * 4, st));
             CK(launch_bin(c->R, c->dp, sa, (int)ns, pl, c->scan_tmp.p, stb, P_<long long>(c->tmpa),
                           P_<long long>(c->tmpb), P_<long long>(c->tmpc), st));
             if ((r = sync1())) return r;
             c->nwide = nw;
-            extra_launches += 6;  // inspect + bin_count, bin_offsets, bin_scatter, list_words, list_offsets
+            extra_launches += 7;  // inspect, mark_wide + bin_count, bin_offsets, bin_scatter, list_words, list_offsets
             if (!h.counters[20]) break;
         }
         // the final wide list: every side inspected with the wide ring (SF_WIDE), for the census
@@ -776,7 +796,8 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     // own kernels: validate, inspect, inspect_block (if escalation on), bin_count, bin_offsets, bin_scatter,
     // list_words, list_offsets, execute per wave, traceback (warp and/or thread variant) per wave, combine_len,
     // combine_total, combine_write
-    S.n_launches = (n > 0 ? 1 + 1 + (esc > 0 ? 1 : 0) + 5 + (int64_t)c->nwaves + tb_launches + 3 + extra_launches : 1);
+    S.n_launches = (n > 0 ? 1 + 1 + (esc > 0 ? 1 : 0) + 5 + (int64_t)c->nwaves + tb_launches + 3 + extra_launches +
+                               (ordered ? 1 : 0) : 1);
     S.n_wide_sides = c->nwide;
     c->have = true;
     return 0;

@@ -54,6 +54,7 @@ constexpr uint32_t SF_EAGER = 1u, SF_OVERFLOW = 2u, SF_RING = 4u, SF_ESCALATE = 
 constexpr uint32_t SF_WIDE = 32u;  // inspected with the wide ring (band wider than the regular ring)
 constexpr uint32_t SF_CHECKFAIL = 64u;  // executor self-check failed (S(i*, j*) mismatch or a store past the reservation)
 constexpr int OPT_NO_EAGER = 1, OPT_NO_TRIM = 2, OPT_NO_BINNING = 4, OPT_NO_BLOCK = 8, OPT_TB_ABOVE_K = 16;
+constexpr int OPT_SELFCHECK_TEST = 1 << 20;  // internal (FASTZ_TEST_SELFCHECK): expect S(i*,j*) + 1, so the check fires
 
 struct DevParams {
     int sv[30];        // sv[5 * code + a] = score(a, code) + O + E: code 0..3 query base, 4 origin column (0), 5 N;

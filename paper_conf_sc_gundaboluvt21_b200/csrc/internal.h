@@ -65,7 +65,11 @@ cudaError_t launch_reverse_packed(const uint32_t* fwd, const uint16_t* fwdn, int
 cudaError_t launch_validate_seeds(const long long* seeds, int n, int tlen, int qlen, long long* bad,
                                   cudaStream_t st);
 int inspector_blocks_per_sm(int R);
-// slist/nlist: inspect only the listed sides (nullptr: all 2n sides); listed sides are flagged SF_WIDE
+// inspector order: predicted side lengths (ungapped walk) sorted longest first into order[nsides]
+size_t order_tmp_bytes(int n);
+cudaError_t launch_order(const Batch& b, const DevParams& P, int nsides, unsigned* keys_in, unsigned* keys_out,
+                         int* vals_in, int* order, void* tmp, size_t tmp_bytes, cudaStream_t st);
+// slist/nlist: inspect the nlist listed sides in that order (nullptr: all 2n sides in index order)
 cudaError_t launch_inspect(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
                            const SideArrays& sa, const ExecPlan& pl, int budget, const int* slist, int nlist,
                            cudaStream_t st);
@@ -83,6 +87,8 @@ size_t lpt_tmp_bytes(int n);
 cudaError_t launch_lpt(const ExecPlan& pl, int nblock, int nexec, const long long* words, long long* keys_in,
                        long long* keys_out, int* vals_in, void* sort_tmp, size_t sort_tmp_bytes, void* scan_tmp,
                        size_t scan_tmp_bytes, cudaStream_t st);
+// flag the listed sides SF_WIDE (after their re-inspection with the wide ring)
+cudaError_t launch_mark_wide(const SideArrays& sa, const int* list, int n, cudaStream_t st);
 // list the sides flagged SF_WIDE (any order) and count them
 cudaError_t launch_wide_list(const SideArrays& sa, int nsides, int* list, int* count, cudaStream_t st);
 // redundant-alignment post-pass (dedup.cu; NEXT-3, reading R14)

@@ -92,6 +92,54 @@ cudaError_t launch_reverse_packed(const uint32_t* fwd, const uint16_t* fwdn, int
     return cudaGetLastError();
 }
 
+// Inspector order (LPT before the inspector; the paper notes the inspector cannot know lengths): a cheap
+// predictor per side -- the extent of an ungapped x-drop walk along the seed's diagonal, capped at PREDICT_CAP
+// bases -- and a radix sort of the sides by it, longest first, so long homologous extensions start early instead
+// of forming a tail at the end of the persistent inspector.  Only the ORDER changes: results are identical.
+constexpr int PREDICT_CAP = 255;
+__global__ void k_predict(Batch b, DevParams P, int nsides, unsigned* keys, int* vals) {
+    const int side = blockIdx.x * blockDim.x + threadIdx.x;
+    if (side >= nsides) return;
+    const int seed = side >> 1;
+    long long tpos = b.seeds[2 * seed], qpos = b.seeds[2 * seed + 1];
+    if (tpos < 0 || tpos > b.tlen || qpos < 0 || qpos > b.qlen) tpos = qpos = 0;
+    const uint32_t *A, *B;
+    long long a0, b0, n;
+    if (side & 1) {
+        A = b.Tf; a0 = tpos; B = b.Qf; b0 = qpos;
+        n = min((long long)b.tlen - tpos, (long long)b.qlen - qpos);
+    } else {
+        A = b.Tr; a0 = b.tlen - tpos; B = b.Qr; b0 = b.qlen - qpos;
+        n = min(tpos, qpos);
+    }
+    n = min(n, (long long)PREDICT_CAP);
+    const int X = 4 * P.OE;  // x-drop of the walk (a few mismatches of headroom)
+    int sc = 0, best = 0, ext = 0;
+    for (int k = 0; k < n; ++k) {
+        const int a = base_at(A, a0 + k), q = base_at(B, b0 + k);
+        sc += P.sv[5 * q + a] - P.OE;
+        if (sc > best) { best = sc; ext = k + 1; }
+        if (sc < best - X) break;
+    }
+    keys[side] = (unsigned)ext;
+    vals[side] = side;
+}
+
+size_t order_tmp_bytes(int n) {
+    size_t bytes = 0;
+    cub::DeviceRadixSort::SortPairsDescending(nullptr, bytes, (const unsigned*)nullptr, (unsigned*)nullptr,
+                                              (const int*)nullptr, (int*)nullptr, n > 0 ? n : 1);
+    return bytes;
+}
+
+cudaError_t launch_order(const Batch& b, const DevParams& P, int nsides, unsigned* keys_in, unsigned* keys_out,
+                         int* vals_in, int* order, void* tmp, size_t tmp_bytes, cudaStream_t st) {
+    if (nsides == 0) return cudaSuccess;
+    k_predict<<<(nsides + 255) / 256, 256, 0, st>>>(b, P, nsides, keys_in, vals_in);
+    size_t bt = tmp_bytes;
+    return cub::DeviceRadixSort::SortPairsDescending(tmp, bt, keys_in, keys_out, vals_in, order, nsides, 0, 9, st);
+}
+
 __global__ void k_validate_seeds(const long long* __restrict__ seeds, int n, int tlen, int qlen, long long* bad) {
     const int s = blockIdx.x * blockDim.x + threadIdx.x;
     if (s >= n) return;
@@ -172,7 +220,6 @@ __device__ __forceinline__ void io_init(SideIO& io, SmemDP& sm, int4* ring, int 
     io.maxsw = 0;
     io.wlim = 0;
     io.xexp = 0;
-    io.written = nullptr;
 }
 
 // eager traceback by lane 0 over the 17x17 corner codes; returns ops (2 bits each, peak -> origin)
@@ -240,9 +287,9 @@ __device__ __forceinline__ void inspect_body(const DevParams& P, const Batch& b,
     io_init(io, sm, ring, rmask, blockIdx.x * WARPS + warp, warp);
     io.eager_max = P.eager_max;
     io.budget = budget;
-    // slist: re-inspection of the sides whose band overflowed the regular ring (wide ring, SF_WIDE)
+    // slist: the order in which to take the sides (predicted-longest first), or the sides whose band overflowed
+    // the regular ring, re-inspected with the wide ring (k_mark_wide flags them afterwards)
     const int nsides = slist ? nlist : 2 * b.nseeds;
-    const uint32_t wide = slist ? SF_WIDE : 0u;
     for (;;) {
         int side = 0;
         if (lane == 0) side = atomicAdd(&pl.counters[0], 1);
@@ -252,7 +299,6 @@ __device__ __forceinline__ void inspect_body(const DevParams& P, const Batch& b,
         setup_side<NM>(b, side, io);
         SideOut o;
         run_side<R, MODE_INSPECT, true, false, NM>(P, io, o);
-        o.flags |= wide;
         __syncwarp();  // eager corner codes (shared memory) written by lanes 0..4 -> read by lane 0
         if (lane == 0) {
             if (o.flags & SF_ESCALATE) {
@@ -347,12 +393,15 @@ __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int
 // Trimmed executor: the DP over [0,i*]x[0,j*] only, writing traceback codes.  Length binning
 // as a schedule: the CTAs first take the long sides (bins >= 3, block per side, strips pipelined
 // across the CTA's warps), then every warp takes short sides (bins 1-2, warp per side), larger bins first.
-// 6 resident CTAs per SM (<= 80 registers): the per-step instruction count of the warp-per-side loop is the same
-// as at its natural 96 registers (5 CTAs), so the extra occupancy is free (SASS: 95 vs 94.5 per 4-cell step)
-#ifndef EXECUTE_MIN_BLOCKS
-#define EXECUTE_MIN_BLOCKS 6
-#endif
+// ptxas's natural 96 registers (5 CTAs per SM).  Capped at 80 (6 CTAs, -DEXECUTE_MIN_BLOCKS=6) the warp-per-side
+// loop keeps its instruction count (SASS 95 vs 94.5 per 4-cell step) but the block-per-side loop grows (111 vs
+// 103) and every config measured slower (tools/config_sweep.py: C2 12.0 vs 10.9 ms, C3 152.7 vs 148.0 ms, C1 124.3
+// vs 120.5 ms; profiles/r2/configs_sweep.jsonl)
+#ifdef EXECUTE_MIN_BLOCKS
 #define EXECUTE_ATTR __launch_bounds__(WARPS * 32, EXECUTE_MIN_BLOCKS)
+#else
+#define EXECUTE_ATTR __launch_bounds__(WARPS * 32)
+#endif
 template <int R, bool NM>
 __global__ void EXECUTE_ATTR k_execute(DevParams P, Batch b, int4* ring, int rmask,
                                                          SideArrays sa, ExecPlan pl, int lo, int hi, int nblock,
@@ -363,6 +412,7 @@ __global__ void EXECUTE_ATTR k_execute(DevParams P, Batch b, int4* ring, int rma
     __shared__ int cur;
     smem_init<NM>(sm, P);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    unsigned long long written = 0;  // code words written by this thread's sides (stats; one atomic at the end)
     for (;;) {  // block phase
         if (threadIdx.x == 0) {
             const int i = lo + atomicAdd(&pl.counters[23], 1);
@@ -387,12 +437,12 @@ __global__ void EXECUTE_ATTR k_execute(DevParams P, Batch b, int4* ring, int rma
         io.codes = out.codes + (pl.woff[side] - base);
         io.stab = out.stab + pl.soff[side];
         io.maxsw = sa.maxsw[side];
-        io.xexp = (P.options & OPT_NO_TRIM) ? INT_MIN : sa.score[side] - P.OE;
-        io.written = (unsigned long long*)(pl.totals + 6);
+        io.xexp = (P.options & OPT_NO_TRIM) ? INT_MIN : sa.score[side] - P.OE + ((P.options & OPT_SELFCHECK_TEST) ? 1 : 0);
         SideOut o;
         run_side<R, MODE_EXEC, false, true, NM>(P, io, o);
         if (threadIdx.x == 0 && (o.flags & SF_RING)) atomicOr(&sa.flags[side], SF_RING);
         if (threadIdx.x == 0 && o.checkfail) atomicAdd(&pl.counters[26], 1);
+        if (threadIdx.x == 0) written += (unsigned long long)o.words;
         __syncthreads();
     }
     SideIO io;
@@ -412,14 +462,15 @@ __global__ void EXECUTE_ATTR k_execute(DevParams P, Batch b, int4* ring, int rma
         io.codes = out.codes + (pl.woff[side] - base);
         io.stab = out.stab + pl.soff[side];
         io.wlim = sa.bound[side];
-        io.xexp = (P.options & OPT_NO_TRIM) ? INT_MIN : sa.score[side] - P.OE;
-        io.written = (unsigned long long*)(pl.totals + 6);
+        io.xexp = (P.options & OPT_NO_TRIM) ? INT_MIN : sa.score[side] - P.OE + ((P.options & OPT_SELFCHECK_TEST) ? 1 : 0);
         SideOut o;
         run_side<R, MODE_EXEC, false, false, NM>(P, io, o);
         if (lane == 0 && (o.flags & SF_RING)) atomicOr(&sa.flags[side], SF_RING);
         if (lane == 0 && o.checkfail) atomicAdd(&pl.counters[26], 1);
+        if (lane == 0) written += (unsigned long long)o.words;
         __syncwarp();
     }
+    if (lane == 0 && written) atomicAdd((unsigned long long*)(pl.totals + 6), written);
 }
 
 // ------------------------------------------------------------------------------------------------- traceback
@@ -641,6 +692,17 @@ __global__ void k_bin_scatter(ExecPlan pl, int nsides) {
     if (bin == 0) return;
     const int pos = atomicAdd(&pl.counters[10 + bin], 1);
     pl.list[pos] = s;
+}
+
+__global__ void k_mark_wide(SideArrays sa, const int* list, int n) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < n) sa.flags[list[i]] |= SF_WIDE;
+}
+
+cudaError_t launch_mark_wide(const SideArrays& sa, const int* list, int n, cudaStream_t st) {
+    if (n <= 0) return cudaSuccess;
+    k_mark_wide<<<(n + 255) / 256, 256, 0, st>>>(sa, list, n);
+    return cudaGetLastError();
 }
 
 __global__ void k_wide_list(SideArrays sa, int nsides, int* list, int* count) {

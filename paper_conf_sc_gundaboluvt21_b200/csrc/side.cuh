@@ -103,7 +103,6 @@ struct SideIO {
                                         // and reported: the executor self-check)
     int xexp;                           // executor: X (= S - O - E) the inspector found at (M, N) = (i*, j*)
                                         // (INT_MIN: not checked -- the untrimmed ablation ends elsewhere)
-    unsigned long long* written;        // executor: code words written (all sides; stats)
 };
 
 struct SideOut {
@@ -596,7 +595,6 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             for (int k = 0; k < R; ++k)
                 if (r0 + k == M) xcap = X[k];
             if (__any_sync(FULL, bad)) flags |= SF_CHECKFAIL;
-            if (lane == 0) atomicAdd(io.written, (unsigned long long)sw);
         }
         const int maxsw_prev = maxsw;
         cum_words += sw;
@@ -614,8 +612,12 @@ __device__ __forceinline__ void run_side(const DevParams& P, const SideIO& io, S
             const int sp = mbj - start > 0 ? mbj - start : 0;
             const int tt2 = tfinal < sp + 31 ? tfinal : sp + 31;
             const int tw = (tt2 / SPW + 1) * 32;
-            bound_words = cum_words - sw + tw;
-            bound_maxsw = imax(maxsw_prev, tw);
+            // strips above: each also covers at most columns [0, j*] (start_k >= 0)
+            const int wj = ((mbj + 31) / SPW + 1) * 32;
+            const long long above = cum_words - sw;
+            const long long cap = (long long)s * wj;
+            bound_words = (above < cap ? above : cap) + tw;
+            bound_maxsw = imax(maxsw_prev < wj ? maxsw_prev : wj, tw);
         }
         bool over = false;
         if (e - start + 4 > rmask) {  // strip wider than the ring: the parked row has been overwritten

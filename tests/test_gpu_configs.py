@@ -44,6 +44,7 @@ def run_bench_config(w):
         st = al.stats()
     finally:
         al.close()
+        torch.cuda.empty_cache()  # the context's pool came from PyTorch's cache: give it back to the driver
     return g, sides, st
 
 

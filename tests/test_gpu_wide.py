@@ -71,3 +71,22 @@ def test_seeds_far_outside_sequences_are_rejected_safely():
     bad, g, o, _ = compare(w.T, w.Q, w.seeds, census=False)
     assert not bad, bad
     assert np.array_equal(good.rec, g.rec) and good.cigar == g.cigar
+
+
+def test_executor_self_check_fires(monkeypatch):
+    """The executor's self-check (recomputed S(i*, j*) == the inspector's peak) is live: with a
+    deliberately wrong expectation (test hook) every executed side fails it and the call returns FASTZ_ECUDA
+    naming the count; without the hook the same batch passes and the stats report no failure."""
+    w = genome.small_pair(92, length=20000, n_seeds=120)
+    with fastz.Aligner(w.T, w.Q) as al:
+        al.extend(w.seeds)
+        st = al.stats()
+        assert st["n_exec_sides"] > 0 and st["n_selfcheck_fail"] == 0
+        assert st["exec_words"] <= st["exec_reserved_words"]
+        monkeypatch.setenv("FASTZ_TEST_SELFCHECK", "1")
+        with pytest.raises(fastz.FastzError) as e:
+            al.extend(w.seeds)
+        assert e.value.status == fastz.FASTZ_ECUDA and "self-check" in str(e.value)
+        assert f"on {st['n_exec_sides']} sides" in str(e.value)
+        monkeypatch.delenv("FASTZ_TEST_SELFCHECK")
+        al.extend(w.seeds)

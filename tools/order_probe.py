@@ -1,6 +1,7 @@
 """Experiment: does the inspector have a long-side tail?  Times fastz_extend_seeds (ms_inspect) on C2 with the
 seeds in their natural (random) order versus the same seeds with the planted long classes first (an oracle-free
-upper bound for any LPT-style inspector ordering, using the generator's class labels)."""
+upper bound for any LPT-style inspector ordering, using the generator's class labels).
+usage: python tools/order_probe.py [config]"""
 import json
 import sys
 
@@ -11,7 +12,8 @@ sys.path.insert(0, ".")
 from paper_conf_sc_gundaboluvt21_b200 import fastz  # noqa: E402
 from synth import genome  # noqa: E402
 
-w = genome.config2()
+cfg = int(sys.argv[1]) if len(sys.argv) > 1 else 2
+w = genome.make(cfg)
 names = w.class_names
 print("classes", names, np.bincount(w.klass), flush=True)
 # longer planted classes first: rank by class index descending (junk = 0 last)
@@ -28,6 +30,7 @@ with fastz.Aligner(w.T, w.Q, torch_alloc=True) as al:
         for _ in range(3):
             al.extend_only(sd)
             ms.append(al.stats()["ms_inspect"])
+        st = al.stats()
         out[name] = ms
-        print(name, ms, flush=True)
+        print(name, ms, "execute", round(st["ms_execute"], 1), "total", round(st["ms_total"], 1), flush=True)
 print(json.dumps(out))
