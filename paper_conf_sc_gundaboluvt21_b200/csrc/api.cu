@@ -15,6 +15,8 @@
 #include <string>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "../../include/fastz.h"
 #include "internal.h"
 
@@ -36,6 +38,20 @@ int fail(int code, const std::string& msg) {
             return fail(_e == cudaErrorMemoryAllocation ? FASTZ_ENOMEM : FASTZ_ECUDA,          \
                         std::string(#x) + ": " + cudaGetErrorString(_e));                       \
     } while (0)
+
+// NVTX range for external profilers (Nsight Systems / Compute): host-side stage markers of fastz_extend_seeds
+// (enqueue + the two host syncs); header-only NVTX v3, a no-op without a profiler attached
+struct Nvtx {
+    bool on = true;
+    explicit Nvtx(const char* name) { nvtxRangePushA(name); }
+    void end() {
+        if (on) nvtxRangePop();
+        on = false;
+    }
+    ~Nvtx() { end(); }
+    Nvtx(const Nvtx&) = delete;
+    Nvtx& operator=(const Nvtx&) = delete;
+};
 
 struct DBuf {
     void* p = nullptr;
@@ -519,6 +535,7 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     if (n < 0 || n > (1 << 29)) return fail(FASTZ_ERANGE, "n must be in [0, 2^29]");
     if (n > 0 && !seeds) return fail(FASTZ_EINVAL, "seeds is NULL");
     CK(cudaSetDevice(c->device));
+    Nvtx range_call("fastz_extend_seeds");
     c->have = false;
     c->n = n;
     const int64_t ns = 2 * n;
@@ -566,6 +583,7 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     Batch b = make_batch(c);
     CK(launch_validate_seeds(b.seeds, b.nseeds, b.tlen, b.qlen, P_<long long>(c->small), st));
     CK(cudaEventRecord(c->ev[1], st));
+    Nvtx range_insp("fastz: inspector");
 
     SideArrays sa = make_sides(c);
     ExecPlan pl = make_plan(c);
@@ -619,6 +637,8 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     }
     if (esc > 0) CK(launch_inspect_block(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, st));
     CK(cudaEventRecord(c->ev[2], st));
+    range_insp.end();
+    Nvtx range_bin("fastz: binning + host sync 1 + pool sizing");
     CK(launch_bin(c->R, c->dp, sa, (int)ns, pl, c->scan_tmp.p, stb, P_<long long>(c->tmpa), P_<long long>(c->tmpb),
                   P_<long long>(c->tmpc), st));
     CK(cudaEventRecord(c->ev[3], st));
@@ -737,6 +757,8 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     Outputs o = make_out(c);
     // executor timing starts here: the host sync + pool sizing above count to the binning stage
     CK(cudaEventRecord(c->ev[7], st));
+    range_bin.end();
+    Nvtx range_exec("fastz: executor + traceback + CIGAR");
     int64_t tb_launches = 0;  // per wave: warp-per-side (list positions < nblock) and thread-per-side launches
     for (size_t w = 0; w < waves.size(); ++w) {
         {
