@@ -19,6 +19,16 @@
  *    twice (after binning, to size the traceback pool -- P:174 "allocation at kernel launch" -- and after
  *    the CIGAR length pass) and otherwise leaves results on the device.
  *  - Scores are int32.  A one-sided peak score >= 2^29 sets FASTZ_FLAG_OVERFLOW on that seed.
+ *  - Self-check: the executor verifies that its recomputed S(i*,j*) equals the inspector's peak and that every
+ *    traceback-code store stays inside the side's reservation; a failure returns FASTZ_ECUDA with the count.
+ *
+ * Environment knobs (experiments and tests; defaults are the measured best): FASTZ_R (rows per lane, 2 or 4;
+ * default 4), FASTZ_INSPECT_ORDER=0 (take sides in seed order instead of predicted-longest first),
+ * FASTZ_ESCALATE_STRIPS (hand sides longer than this many strips to the block-per-side inspector; default off),
+ * FASTZ_BLOCK_BIN (smallest executor bin run block per side; default 3), FASTZ_POOL_MB (traceback-pool budget;
+ * default 80% of free memory), FASTZ_RING_ENTRIES (boundary-ring entries per warp; wider bands take the wide
+ * ring), FASTZ_L2_PERSIST=1 (boundary rings in an L2 persisting window during the inspector), FASTZ_SEED_HIT_CAP
+ * (seeding scratch), FASTZ_TEST_SELFCHECK=1 (test hook: makes the executor self-check fail).
  */
 #ifndef FASTZ_H
 #define FASTZ_H

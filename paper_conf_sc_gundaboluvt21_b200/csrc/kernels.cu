@@ -93,10 +93,20 @@ cudaError_t launch_reverse_packed(const uint32_t* fwd, const uint16_t* fwdn, int
 }
 
 // Inspector order (LPT before the inspector; the paper notes the inspector cannot know lengths): a cheap
-// predictor per side -- the extent of an ungapped x-drop walk along the seed's diagonal, capped at PREDICT_CAP
-// bases -- and a radix sort of the sides by it, longest first, so long homologous extensions start early instead
-// of forming a tail at the end of the persistent inspector.  Only the ORDER changes: results are identical.
-constexpr int PREDICT_CAP = 255;
+// predictor per side and a radix sort of the sides by it, longest first, so long homologous extensions start early
+// instead of forming a tail at the end of the persistent inspector.  Only the ORDER changes: results are identical.
+// Predictor: an x-drop walk along the seed's diagonal that may step over up to PREDICT_SHIFTS one-base indels
+// (when the walk drops X below its best, it resumes from the best point on the better of the two neighbouring
+// diagonals, judged on the next 8 bases), capped at PREDICT_CAP bases: chance seeds stop after a few bases, short
+// homology at its end, long homology saturates.
+constexpr int PREDICT_CAP = 2047, PREDICT_SHIFTS = 16, PREDICT_BITS = 11;
+__device__ __forceinline__ int predict_score8(const DevParams& P, const uint32_t* A, long long a0, long long na,
+                                              const uint32_t* B, long long b0, long long nb, long long i, long long j) {
+    int sc = 0;
+    for (int k = 0; k < 8 && i + k < na && j + k < nb; ++k)
+        sc += P.sv[5 * base_at(B, b0 + j + k) + base_at(A, a0 + i + k)] - P.OE;
+    return sc;
+}
 __global__ void k_predict(Batch b, DevParams P, int nsides, unsigned* keys, int* vals) {
     const int side = blockIdx.x * blockDim.x + threadIdx.x;
     if (side >= nsides) return;
@@ -104,24 +114,40 @@ __global__ void k_predict(Batch b, DevParams P, int nsides, unsigned* keys, int*
     long long tpos = b.seeds[2 * seed], qpos = b.seeds[2 * seed + 1];
     if (tpos < 0 || tpos > b.tlen || qpos < 0 || qpos > b.qlen) tpos = qpos = 0;
     const uint32_t *A, *B;
-    long long a0, b0, n;
+    long long a0, b0, na, nb;
     if (side & 1) {
         A = b.Tf; a0 = tpos; B = b.Qf; b0 = qpos;
-        n = min((long long)b.tlen - tpos, (long long)b.qlen - qpos);
+        na = (long long)b.tlen - tpos; nb = (long long)b.qlen - qpos;
     } else {
         A = b.Tr; a0 = b.tlen - tpos; B = b.Qr; b0 = b.qlen - qpos;
-        n = min(tpos, qpos);
+        na = tpos; nb = qpos;
     }
-    n = min(n, (long long)PREDICT_CAP);
+    na = min(na, (long long)PREDICT_CAP);
     const int X = 4 * P.OE;  // x-drop of the walk (a few mismatches of headroom)
-    int sc = 0, best = 0, ext = 0;
-    for (int k = 0; k < n; ++k) {
-        const int a = base_at(A, a0 + k), q = base_at(B, b0 + k);
-        sc += P.sv[5 * q + a] - P.OE;
-        if (sc > best) { best = sc; ext = k + 1; }
-        if (sc < best - X) break;
+    int sc = 0, best = 0, shifts = 0;
+    long long i = 0, j = 0, bi = 0, bj = 0;
+    while (i < na && j < nb) {
+        sc += P.sv[5 * base_at(B, b0 + j) + base_at(A, a0 + i)] - P.OE;
+        ++i;
+        ++j;
+        if (sc > best) {
+            best = sc;
+            bi = i;
+            bj = j;
+        } else if (sc < best - X) {
+            if (++shifts > PREDICT_SHIFTS) break;
+            const int sd = predict_score8(P, A, a0, na, B, b0, nb, bi + 1, bj);  // skip a target base
+            const int si = predict_score8(P, A, a0, na, B, b0, nb, bi, bj + 1);  // skip a query base
+            // resume only if a neighbouring diagonal clearly continues (~6 of 8 bases matching): chance
+            // seeds stop at their first drop, so the walk costs them a few dozen base reads
+            const int need = 3 * (P.sv[0] - P.OE);  // 3 x sub(A, A)
+            if (sd < need && si < need) break;
+            i = sd >= si ? bi + 1 : bi;
+            j = sd >= si ? bj : bj + 1;
+            sc = best - P.OE;
+        }
     }
-    keys[side] = (unsigned)ext;
+    keys[side] = (unsigned)(bi < PREDICT_CAP ? bi : PREDICT_CAP);
     vals[side] = side;
 }
 
@@ -137,7 +163,8 @@ cudaError_t launch_order(const Batch& b, const DevParams& P, int nsides, unsigne
     if (nsides == 0) return cudaSuccess;
     k_predict<<<(nsides + 255) / 256, 256, 0, st>>>(b, P, nsides, keys_in, vals_in);
     size_t bt = tmp_bytes;
-    return cub::DeviceRadixSort::SortPairsDescending(tmp, bt, keys_in, keys_out, vals_in, order, nsides, 0, 9, st);
+    return cub::DeviceRadixSort::SortPairsDescending(tmp, bt, keys_in, keys_out, vals_in, order, nsides, 0,
+                                                     PREDICT_BITS, st);
 }
 
 __global__ void k_validate_seeds(const long long* __restrict__ seeds, int n, int tlen, int qlen, long long* bad) {
