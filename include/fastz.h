@@ -220,6 +220,10 @@ typedef struct {
     int64_t exec_reserved_words;  /* traceback-pool words reserved for the executor (>= exec_words) */
     int64_t n_selfcheck_fail;     /* executor self-check failures: S(i*,j*) != inspector score, or code words
                                      outside a side's reservation (always 0; nonzero -> FASTZ_ECUDA) */
+    int64_t n_packed_sides;       /* sides given to the packed (two per warp, 16-bit) inspector */
+    int64_t n_long_sides;         /* sides predicted long, inspected first by the 32-bit inspector */
+    int64_t n_redo_sides;         /* packed sides that reached the 16-bit value cap and were re-inspected in 32 bits
+                                     (results never depend on which inspector ran a side) */
 } fastz_stats;
 int fastz_get_stats(fastz_ctx *c, fastz_stats *s);
 

@@ -10,7 +10,7 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libfastz.so")
 SOURCES = ["api.cu", "kernels.cu", "intpeak.cu", "seeds.cu", "dedup.cu"]
-HEADERS = ["dp.cuh", "side.cuh", "internal.h"]
+HEADERS = ["dp.cuh", "side.cuh", "pair.cuh", "internal.h"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",
          "-Xcompiler", "-fPIC", "-shared", "-Xptxas", "-warn-spills", "-diag-suppress", "177"]

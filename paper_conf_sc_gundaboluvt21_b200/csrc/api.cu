@@ -73,12 +73,18 @@ struct fastz_ctx {
     DBuf seeds, score, ti, qj, flags, eops, bound, maxsw, esc, nstrip;
     DBuf woff, soff, roff, bin, list, counters, totals, tmpa, tmpb, tmpc, scan_tmp, wl, wlo;
     DBuf codes, stab, runs, nruns, ciglen, cigar, recs, cells, ring, small, wide, ring2, lpt_tmp, order_tmp, order_buf;
+    DBuf ring_pair, redo;  // packed inspector (pair.cuh): two rings of int2 per warp slot; abandoned sides
     // seeding (fastz_find_hsps)
     DBuf s_kin, s_kout, s_pin, s_pout, s_start, s_cnt, s_off, s_hits, s_hsp, s_keep, s_sel, s_list, s_list2,
         s_k1, s_k2, s_i1, s_i2, s_flag, s_pos, s_out, s_anch, s_tmp;
     // redundant-alignment post-pass (fastz_mark_redundant)
     DBuf r_k1, r_k2, r_i1, r_i2, r_box, r_sc, r_red, r_tmp, r_cnt;
     int R = 4, grid = 0, nslots = 0, rmask = 0;
+    // packed inspector: launch grid (0 = not built for this context), constants, whether the parameters admit it
+    int grid_pair = 0, grid_mixed = 0;
+    PairParams pq{};
+    bool pair_params_ok = false;
+    int64_t n_pair_sides = 0, n_redo_sides = 0, n_long_sides = 0;
     // wide ring of the last batch (sides whose explored band overflowed `ring`): grid2 CTAs x WARPS slots of
     // rmask2 + 1 entries; nwide sides listed in `wide`
     int grid2 = 0, rmask2 = 0, nwide = 0;
@@ -87,6 +93,9 @@ struct fastz_ctx {
     bool have = false;
     fastz_stats stats{};
     cudaEvent_t ev[8] = {};
+    // second stream: the 32-bit inspector of the predicted-long sides runs beside the packed inspector
+    cudaStream_t side_stream = nullptr;
+    cudaEvent_t fork_ev = nullptr, join_ev = nullptr;
     bool ev_ok = false;
 };
 
@@ -243,6 +252,7 @@ ExecPlan make_plan(fastz_ctx* c) {
     p.wl = P_<long long>(c->wl);
     p.wlo = P_<long long>(c->wlo);
     p.wide = P_<int>(c->wide);
+    p.redo = P_<int>(c->redo);
     return p;
 }
 
@@ -256,6 +266,60 @@ Outputs make_out(fastz_ctx* c) {
     o.cigar = P_<char>(c->cigar);
     o.recs = c->recs.p;
     return o;
+}
+
+// Constants of the packed inspector (pair.cuh).  Stored 16-bit value = true + Z.
+// Every quantity of a cell must stay in [0, 65535] without any cross-half carry:
+//   dead X = NEG_b = max(Y, O+E, E)   (so S - Y, S - OE and D - E never go below 0)
+//   NEG_t  = -(Y + 2 + max(sub + OE)) (a cell fed only by dead cells stays below every threshold >= -(Y+1))
+//   BIG_b  = NEG_b + 32767            (rows beyond M / columns beyond N; S - W + 0x8000 stays in 16 bits)
+//   a side is abandoned (redone in 32 bits) once its peak X reaches limX: values never exceed BIG_b before that
+// Returns false when the parameters leave no useful score range (the 32-bit inspector then takes every side).
+bool pair_params(const DevParams& d, PairParams& q) {
+    int svmax = INT_MIN, svmin = INT_MAX;
+    for (int code = 0; code < 5; ++code)
+        for (int a = 0; a < 4; ++a) {
+            svmax = std::max(svmax, d.sv[5 * code + a]);
+            svmin = std::min(svmin, d.sv[5 * code + a]);
+        }
+    if (d.Y < 0 || d.E < 0 || d.OE < 0 || svmin < 0) return false;
+    const int64_t negb = std::max<int64_t>(std::max<int64_t>(d.Y, d.OE), std::max<int64_t>(d.E, 1));
+    if (negb > 30000 || svmax > 4000) return false;
+    const int64_t bigb = negb + 32767;
+    const int64_t negt = -((int64_t)d.Y + 2 + svmax);
+    const int64_t Z = negb - negt;
+    const int64_t bigt = bigb - Z;
+    const int64_t sm = std::max<int64_t>(0, svmax - d.OE);  // largest per-step growth of S
+    const int64_t limt = bigt - d.OE - 4 * sm - 64;        // peak X (true) that abandons the side
+    if (limt < 2000) return false;
+    q.Z = (unsigned)Z;
+    q.NEGb = (unsigned)negb;
+    q.BIGb = (unsigned)bigb;
+    q.mE2 = ((65536u - (unsigned)d.E) & 0xffffu) * 0x10001u;
+    q.mY2 = 0u - (unsigned)d.Y * 0x10001u;
+    q.mOE2 = 0u - (unsigned)d.OE * 0x10001u;
+    q.limX = (unsigned)(limt + Z);
+    q.WoutT = -d.Y - 1;
+    const char* e = getenv("FASTZ_PAIR_ESCAPE");
+    q.esc_strips = e ? std::max(1, atoi(e)) : 16;
+    return true;
+}
+
+// the packed inspector takes this batch: parameters admit it, 4 rows per lane, no N (the N-aware tables are
+// 32-bit only), and enough sides to keep every warp busy -- a batch with fewer sides than ~16 per warp is bound by
+// its longest sides, which a packed warp steps ~2x slower (FASTZ_PAIR=0 never, =2 always, e.g. for tests)
+bool use_pair(const fastz_ctx* c, const Batch& b, int64_t ns) {
+    const char* e = getenv("FASTZ_PAIR");
+    const int mode = e ? atoi(e) : 1;
+    if (mode == 0 || !c->pair_params_ok || c->R != 4 || b.TfN || b.TrN || b.QfN || b.QrN) return false;
+    return mode == 2 || ns >= 16 * (int64_t)c->grid_mixed * WARPS;
+}
+
+// predicted length (k_predict's ungapped walk, bases) from which a side goes to the 32-bit inspector first
+unsigned pair_long_threshold() {
+    const char* e = getenv("FASTZ_PAIR_LONG");
+    const long v = e ? atol(e) : 96;
+    return (unsigned)(v < 0 ? 0 : v);
 }
 
 int ensure_ring(fastz_ctx* c) {
@@ -321,11 +385,15 @@ void fastz_destroy(fastz_ctx* c) {
                     &c->small, &c->s_kin, &c->s_kout, &c->s_pin, &c->s_pout, &c->s_start, &c->s_cnt, &c->s_off,
                     &c->s_hits, &c->s_hsp, &c->s_keep, &c->s_sel, &c->s_list, &c->s_list2, &c->s_k1, &c->s_k2,
                     &c->s_i1, &c->s_i2, &c->s_flag, &c->s_pos, &c->s_out, &c->s_anch, &c->s_tmp,
-                    &c->r_k1, &c->r_k2, &c->r_i1, &c->r_i2, &c->r_box, &c->r_sc, &c->r_red, &c->r_tmp, &c->r_cnt};
+                    &c->r_k1, &c->r_k2, &c->r_i1, &c->r_i2, &c->r_box, &c->r_sc, &c->r_red, &c->r_tmp, &c->r_cnt,
+                    &c->ring_pair, &c->redo};
     for (DBuf* b : bufs) dfree(c, *b);
     if (c->ev_ok)
         for (auto& e : c->ev) cudaEventDestroy(e);
     if (c->own_stream && c->stream) cudaStreamDestroy(c->stream);
+    if (c->side_stream) cudaStreamDestroy(c->side_stream);
+    if (c->fork_ev) cudaEventDestroy(c->fork_ev);
+    if (c->join_ev) cudaEventDestroy(c->join_ev);
     delete c;
 }
 
@@ -379,6 +447,7 @@ int ctx_begin(const fastz_params* p, int64_t tlen, int64_t qlen, int device, voi
     c->dp.OE = p->gap_open + p->gap_extend;
     c->dp.K = p->gapped_threshold;
     c->dp.eager_max = p->eager_max;
+    c->pair_params_ok = pair_params(c->dp, c->pq);
     c->tlen = (int)tlen;
     c->qlen = (int)qlen;
     *out = c;
@@ -392,6 +461,8 @@ void ctx_finish(fastz_ctx* c) {
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, c->device);
     c->grid = sms * inspector_blocks_per_sm(c->R);
     c->nslots = c->grid * WARPS;
+    c->grid_pair = sms * pair_blocks_per_sm();
+    c->grid_mixed = sms * mixed_blocks_per_sm();
     // per-warp boundary ring: the widest explored band is bounded by the query side length; capped (wider
     // bands take the wide ring, fastz_extend_seeds)
     int64_t want = std::max<int64_t>(std::max<int64_t>(c->tlen, c->qlen) + 64, 1024);
@@ -551,6 +622,7 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     AL(bound, std::max<int64_t>(ns, 1) * 8);
     AL(maxsw, std::max<int64_t>(ns, 1) * 4);
     AL(esc, std::max<int64_t>(ns, 1) * 4);
+    AL(redo, std::max<int64_t>(ns, 1) * 4);
     AL(nstrip, std::max<int64_t>(ns, 1) * 4);
     AL(woff, std::max<int64_t>(ns, 1) * 8);
     AL(soff, std::max<int64_t>(ns, 1) * 8);
@@ -566,7 +638,7 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     AL(wide, std::max<int64_t>(ns, 1) * 4);
     AL(ciglen, std::max<int64_t>(2 * n, 1) * 8);
     AL(recs, std::max<int64_t>(n, 1) * sizeof(fastz_alignment));
-    AL(counters, 64 * 4);
+    AL(counters, 96 * 4);
     AL(totals, 8 * 8);
     AL(small, 64);
     const size_t stb = scan_tmp_bytes((int)std::max<int64_t>(ns, 1));
@@ -576,7 +648,7 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     if (n > 0)
         CK(cudaMemcpyAsync(c->seeds.p, seeds, (size_t)n * 16,
                            seeds_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, st));
-    CK(cudaMemsetAsync(c->counters.p, 0, 64 * 4, st));
+    CK(cudaMemsetAsync(c->counters.p, 0, 96 * 4, st));
     CK(cudaMemsetAsync(c->totals.p, 0, 8 * 8, st));
     long long init = LLONG_MAX;
     CK(cudaMemcpyAsync(c->small.p, &init, sizeof(init), cudaMemcpyHostToDevice, st));
@@ -627,8 +699,93 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
                         c->order_tmp.cap, st));
         order = P_<int>(c->order_buf);
     }
-    CK(launch_inspect(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, esc > 0 ? esc : INT_MAX,
-                      order, ordered ? (int)ns : 0, st));
+    int64_t pair_launches = 0;
+    bool pair_run = false;
+    c->n_pair_sides = c->n_redo_sides = c->n_long_sides = 0;
+    if (use_pair(c, b, ns)) {
+        // Packed inspector (pair.cuh, kernels.cu k_inspect_mixed).  The sides predicted long (k_predict >=
+        // FASTZ_PAIR_LONG bases: the head of the order, counted by k_split) run in k_inspect on a second stream,
+        // concurrently; the rest run two per warp in 16-bit halves, and the sides the packed inspector abandons
+        // (value cap, too many strips) are re-inspected by its own 32-bit path.  The eager walk of the packed sides
+        // follows (k_eager).
+        int nlong = 0;
+        if (ordered) {
+            CK(launch_split(reinterpret_cast<unsigned*>(P_<long long>(c->tmpa)) + ns, (int)ns, pair_long_threshold(),
+                            P_<int>(c->counters) + 28, st));
+            CK(cudaMemcpyAsync(&nlong, P_<int>(c->counters) + 28, 4, cudaMemcpyDeviceToHost, st));
+            CK(cudaStreamSynchronize(st));
+            pair_launches += 1;
+        }
+        CK(cudaMemsetAsync(c->redo.p, 0xff, (size_t)ns * 4, st));
+        const size_t rb = (size_t)c->grid_mixed * WARPS * (size_t)(c->rmask + 1) * sizeof(int4);
+        AL(ring_pair, rb);
+        // diagnostics (FASTZ_PAIR_DEBUG=1): per packed side {cycles, strips, steps, redo} -> stderr summary
+        long long* dbg = nullptr;
+        const bool pdebug = getenv("FASTZ_PAIR_DEBUG") != nullptr;
+        if (pdebug) {
+            AL(wl, (std::max<int64_t>(ns, 1) + (int64_t)c->grid_mixed * WARPS) * 32);
+            dbg = P_<long long>(c->wl);
+            CK(cudaMemsetAsync(dbg, 0, (size_t)(ns + (int64_t)c->grid_mixed * WARPS) * 32, st));
+        }
+        if (nlong > 0) {
+            if (!c->side_stream) {
+                CK(cudaStreamCreateWithFlags(&c->side_stream, cudaStreamNonBlocking));
+                CK(cudaEventCreateWithFlags(&c->fork_ev, cudaEventDisableTiming));
+                CK(cudaEventCreateWithFlags(&c->join_ev, cudaEventDisableTiming));
+            }
+            CK(cudaEventRecord(c->fork_ev, st));
+            CK(cudaStreamWaitEvent(c->side_stream, c->fork_ev, 0));
+            CK(launch_inspect(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, esc > 0 ? esc : INT_MAX,
+                              order, nlong, c->side_stream));
+            CK(cudaEventRecord(c->join_ev, c->side_stream));
+            pair_launches += 1;
+        }
+        CK(launch_inspect_mixed(c->grid_mixed, c->dp, c->pq, b, P_<int4>(c->ring_pair), c->rmask, sa, pl,
+                                ordered ? order : nullptr, (int)ns, nlong, 0, INT_MAX, dbg, st));
+        if (nlong > 0) CK(cudaStreamWaitEvent(st, c->join_ev, 0));
+        CK(launch_eager(c->dp, b, sa, (int)ns, st));
+        pair_launches += 2;
+        pair_run = true;
+        if (pdebug) {
+            const int64_t nw = (int64_t)c->grid_mixed * WARPS;
+            std::vector<long long> d((size_t)(ns + nw) * 4);
+            CK(cudaMemcpyAsync(d.data(), dbg, (size_t)(ns + nw) * 32, cudaMemcpyDeviceToHost, st));
+            CK(cudaStreamSynchronize(st));
+            {
+                double p1 = 0, p2 = 0, ex = 0, mx1 = 0, mx2 = 0, mxe = 0, n32 = 0;
+                for (int64_t w = 0; w < nw; ++w) {
+                    const long long* q = &d[(size_t)(4 * ns + 4 * w)];
+                    p1 += q[0]; p2 += q[1]; ex += q[2]; n32 += q[3];
+                    mx1 = std::max(mx1, (double)q[0]); mx2 = std::max(mx2, (double)q[1]); mxe = std::max(mxe, (double)q[2]);
+                }
+                fprintf(stderr, "mixed debug: %lld warps; cycles to end of phase 1 mean %.0f max %.0f, phase 2 mean %.0f "
+                        "max %.0f, exit mean %.0f max %.0f; 32-bit sides %.0f\n", (long long)nw, p1 / nw, mx1, p2 / nw,
+                        mx2, ex / nw, mxe, n32);
+            }
+            std::vector<int64_t> idx;
+            double cyc = 0, steps = 0;
+            int64_t nred = 0, npk = 0;
+            for (int64_t k = 0; k < ns; ++k)
+                if (d[4 * k]) {
+                    idx.push_back(k);
+                    cyc += (double)d[4 * k];
+                    steps += (double)d[4 * k + 2];
+                    nred += d[4 * k + 3];
+                    ++npk;
+                }
+            std::sort(idx.begin(), idx.end(), [&](int64_t a, int64_t b2) { return d[4 * a] > d[4 * b2]; });
+            fprintf(stderr, "pair debug: %lld packed sides, %lld redo, mean %.0f cycles, mean %.1f steps\n",
+                    (long long)npk, (long long)nred, cyc / std::max<int64_t>(npk, 1), steps / std::max<int64_t>(npk, 1));
+            for (size_t k = 0; k < idx.size() && k < 8; ++k) {
+                const int64_t s2 = idx[k];
+                fprintf(stderr, "  side %lld: %lld cycles, %lld strips, %lld steps, redo %lld\n", (long long)s2,
+                        d[4 * s2], d[4 * s2 + 1], d[4 * s2 + 2], d[4 * s2 + 3]);
+            }
+        }
+    } else {
+        CK(launch_inspect(c->R, c->grid, c->dp, b, P_<int4>(c->ring), c->rmask, sa, pl, esc > 0 ? esc : INT_MAX,
+                          order, ordered ? (int)ns : 0, st));
+    }
     if (persist) {
         cudaStreamAttrValue a{};
         a.accessPolicyWindow.num_bytes = 0;
@@ -646,7 +803,7 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     // host sync 1: sizes of the executor's traceback pool
     struct {
         long long totals[5];
-        int counters[26];
+        int counters[36];
         long long bad;
     } h;
     auto sync1 = [&]() -> int {
@@ -657,6 +814,11 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
         return 0;
     };
     if ((r = sync1())) return r;
+    if (pair_run) {
+        c->n_long_sides = ordered ? h.counters[28] : 0;
+        c->n_pair_sides = ns - c->n_long_sides;
+        c->n_redo_sides = h.counters[30];
+    }
     if (h.bad != LLONG_MAX) return fail(FASTZ_ERANGE, "seed " + std::to_string(h.bad) + " lies outside the sequences");
     // Sides whose explored band outgrew the per-warp boundary ring (possible only for very large Y or long
     // indel-rich alignments; the y-drop rule itself has no width limit) are re-inspected with a ring 4x
@@ -684,10 +846,10 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
             // re-inspect the listed sides (wide list -> tmp copy, since binning rebuilds it)
             int* wl = P_<int>(c->tmpc);
             CK(cudaMemcpyAsync(wl, c->wide.p, (size_t)nw * 4, cudaMemcpyDeviceToDevice, st));
-            CK(cudaMemsetAsync(c->counters.p, 0, 64 * 4, st));
+            CK(cudaMemsetAsync(c->counters.p, 0, 96 * 4, st));
             CK(launch_inspect(c->R, c->grid2, c->dp, b, P_<int4>(c->ring2), c->rmask2, sa, pl, INT_MAX, wl, nw, st));
             CK(launch_mark_wide(sa, wl, nw, st));
-            CK(cudaMemsetAsync(c->counters.p, 0, 64 * 4, st));
+            CK(cudaMemsetAsync(c->counters.p, 0, 96 * 4, st));
             CK(launch_bin(c->R, c->dp, sa, (int)ns, pl, c->scan_tmp.p, stb, P_<long long>(c->tmpa),
                           P_<long long>(c->tmpb), P_<long long>(c->tmpc), st));
             if ((r = sync1())) return r;
@@ -819,8 +981,11 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
     // list_words, list_offsets, execute per wave, traceback (warp and/or thread variant) per wave, combine_len,
     // combine_total, combine_write
     S.n_launches = (n > 0 ? 1 + 1 + (esc > 0 ? 1 : 0) + 5 + (int64_t)c->nwaves + tb_launches + 3 + extra_launches +
-                               (ordered ? 1 : 0) : 1);
+                               (ordered ? 1 : 0) + pair_launches : 1);
     S.n_wide_sides = c->nwide;
+    S.n_packed_sides = c->n_pair_sides;
+    S.n_long_sides = c->n_long_sides;
+    S.n_redo_sides = c->n_redo_sides;
     c->have = true;
     return 0;
 }

@@ -53,6 +53,7 @@ constexpr int SUBTAB_INTS = SubTab<true>::INTS;  // shared allocation (the large
 constexpr uint32_t SF_EAGER = 1u, SF_OVERFLOW = 2u, SF_RING = 4u, SF_ESCALATE = 8u, SF_NOTB = 16u;
 constexpr uint32_t SF_WIDE = 32u;  // inspected with the wide ring (band wider than the regular ring)
 constexpr uint32_t SF_CHECKFAIL = 64u;  // executor self-check failed (S(i*, j*) mismatch or a store past the reservation)
+constexpr uint32_t SF_PAIR = 1u << 20;  // inspected by the packed kernel (pair.cuh); k_eager clears it after the eager walk
 constexpr int OPT_NO_EAGER = 1, OPT_NO_TRIM = 2, OPT_NO_BINNING = 4, OPT_NO_BLOCK = 8, OPT_TB_ABOVE_K = 16;
 constexpr int OPT_SELFCHECK_TEST = 1 << 20;  // internal (FASTZ_TEST_SELFCHECK): expect S(i*,j*) + 1, so the check fires
 

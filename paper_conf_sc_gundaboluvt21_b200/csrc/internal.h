@@ -38,12 +38,14 @@ struct ExecPlan {
                          // occupy list[0, totals[4])
     int* counters;       // [0] inspector queue, [1] executor warp queue, [2..8] bin counts, [10..16] bin cursors,
                          // [20] ring overflow, [21] escalated sides, [22] block inspector queue,
-                         // [23] executor block queue, [24] wide (ring-overflow) sides
+                         // [23] executor block queue, [24] wide (ring-overflow) sides, [28] predicted-long sides
+                         // (32-bit inspector), [30] packed-inspector redo sides
     long long* totals;   // [0] words, [1] strips, [2] runs, [3] n_exec, [4] n_exec_block
     int* esc;            // escalated sides (inspector -> block inspector)
     long long* wl;       // executor words in list order (scratch)
     long long* wlo;      // exclusive scan of wl: pool offset of list position i
     int* wide;           // sides whose band overflowed the regular ring (counters[24] of them)
+    int* redo;           // sides the packed inspector abandoned (value cap), re-inspected in 32 bits (counters[30])
 };
 
 struct Outputs {
@@ -54,6 +56,20 @@ struct Outputs {
     long long* cig_len;  // per seed CIGAR length, then exclusive-scanned in place into offsets
     char* cigar;
     void* recs;          // fastz_alignment[n]
+};
+
+// Packed inspector constants (pair.cuh): stored 16-bit value = true value + Z
+struct PairParams {
+    unsigned Z;      // bias: stored = true + Z
+    unsigned NEGb;   // dead X (and D / I never fall below it)
+    unsigned BIGb;   // threshold of rows beyond M and columns beyond N: nothing there is live
+    unsigned mE2;    // per-half (-E) mod 2^16
+    unsigned mY2;    // -(Y * 0x10001): 32-bit add, no borrow since every S >= NEG_b >= Y
+    unsigned mOE2;   // -(OE * 0x10001)
+    unsigned limX;   // value cap: a half whose peak X (stored) reaches limX is redone in 32 bits
+    int WoutT;       // W left of column 0 (true value, -(Y+1))
+    int esc_strips;  // a packed side still running after this many strips is redone in 32 bits (long sides must
+                     // not run packed: a lone packed warp steps ~2x slower than a 32-bit one)
 };
 
 int pick_R();  // rows per lane (FASTZ_R env: 2, 4 or 8; default 4)
@@ -73,6 +89,24 @@ cudaError_t launch_order(const Batch& b, const DevParams& P, int nsides, unsigne
 cudaError_t launch_inspect(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
                            const SideArrays& sa, const ExecPlan& pl, int budget, const int* slist, int nlist,
                            cudaStream_t st);
+// packed inspector: sides slist[0, nsides) (all sides when slist is null), two per warp; abandoned sides go to
+// pl.redo (counters[30]).  pair_blocks_per_sm: occupancy of the packed kernel.
+int pair_blocks_per_sm();
+// packed inspection (kernels.cu k_inspect_mixed): order[0, n1) in its 32-bit path (queue counters[35]; n1 = 0 when
+// a concurrent k_inspect takes the predicted-long head order[0, nlong)), order[nlong, nsides) packed two per warp
+// (queue counters[32]), and the sides the packed phase abandons (pl.redo, pre-set to -1; pushes counters[30],
+// claims counters[34]) in its 32-bit path.  dbg: optional diagnostics buffer (FASTZ_PAIR_DEBUG).
+int mixed_blocks_per_sm();
+cudaError_t launch_inspect_mixed(int grid, const DevParams& P, const PairParams& Q, const Batch& b, int4* ring,
+                                 int rmask, const SideArrays& sa, const ExecPlan& pl, const int* order, int nsides,
+                                 int nlong, int n1, int budget, long long* dbg, cudaStream_t st);
+cudaError_t launch_inspect_pair(int grid, const DevParams& P, const PairParams& Q, const Batch& b, int2* ring,
+                                int rmask, const SideArrays& sa, const ExecPlan& pl, const int* slist, int nsides,
+                                cudaStream_t st);
+// *count = number of sorted (descending) prediction keys >= thr: the sides the 32-bit inspector takes first
+cudaError_t launch_split(const unsigned* keys_desc, int n, unsigned thr, int* count, cudaStream_t st);
+// eager walk of the packed inspector's sides whose peak lies in the 17x17 corner; clears SF_PAIR
+cudaError_t launch_eager(const DevParams& P, const Batch& b, const SideArrays& sa, int nsides, cudaStream_t st);
 cudaError_t launch_inspect_block(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
                                  const SideArrays& sa, const ExecPlan& pl, cudaStream_t st);
 int escalate_strips();  // FASTZ_ESCALATE_STRIPS (default 16; 0 disables block-per-side inspection)

@@ -364,6 +364,304 @@ __global__ void __maxnreg__(INSPECT_N_MAXREG) k_inspect_n(DevParams P, Batch b, 
     inspect_body<R, true>(P, b, ring, rmask, sa, pl, budget, slist, nlist);
 }
 
+// ------------------------------------------------------------------------------------------- packed inspector
+}  // namespace fz
+#include "pair.cuh"
+namespace fz {
+// Two sides per warp in 16-bit halves (pair.cuh).  Persistent: each half of each warp pops sides from the queue
+// (slist[0, ns) in order, or all sides when slist is null).
+struct SmemPair {
+    alignas(16) int subtab[PSUB_INTS];
+    PairWarp w[WARPS];
+};
+
+template <int R>
+__global__ void __launch_bounds__(WARPS * 32) k_inspect_pair(DevParams P, PairParams Q, Batch b, int2* ring,
+                                                             int rmask, SideArrays sa, ExecPlan pl, const int* slist,
+                                                             int ns) {
+    __shared__ SmemPair sm;
+    // tables L (low halves) and H (high halves): entry (code, a0, a1), 16 replicas of 8 bytes
+    for (int idx = threadIdx.x; idx < PSUB_INTS / 2; idx += blockDim.x) {
+        const int tab = idx / (PSUB_TAB / 8), rem = idx % (PSUB_TAB / 8);
+        const int e = rem / SUBTAB_REP, code = e / 16, a0 = (e / 4) % 4, a1 = e % 4;
+        const unsigned v0 = (unsigned)P.sv[5 * code + a0], v1 = (unsigned)P.sv[5 * code + a1];
+        sm.subtab[2 * idx] = (int)(tab ? v0 << 16 : v0);
+        sm.subtab[2 * idx + 1] = (int)(tab ? v1 << 16 : v1);
+    }
+    for (int idx = threadIdx.x; idx < WARPS * (PCP_RING + BLK); idx += blockDim.x)
+        sm.w[idx / (PCP_RING + BLK)].co[idx % (PCP_RING + BLK)] = make_int2(4 * PSUB_CODE, 4 * PSUB_CODE);
+    __syncthreads();
+    const int warp = threadIdx.x >> 5;
+    int2* rb = ring + (size_t)(blockIdx.x * WARPS + warp) * 2 * (size_t)(rmask + 1);
+    run_pairs<R>(P, Q, b, rb, rmask, sa, pl, &sm.w[warp], (unsigned)__cvta_generic_to_shared(sm.subtab), slist, ns,
+                 &pl.counters[0]);
+}
+
+// One persistent launch for the whole inspection when the packed inspector is on (no tails between phases):
+//   phase 1: the predicted-long sides order[0, nlong) one per warp in the 32-bit inspector (inline eager walk);
+//   phase 2: the other sides two per warp in the packed inspector (queue counters[32]);
+//   then the sides phase 2 abandoned (value cap, or too many strips: pl.redo, pre-set to -1, counters[30] pushes,
+//   counters[34] claims), in the 32-bit inspector, by whichever warp claims them first (see below).
+// The 32-bit path reads the packed tables' low-half table (the same layout as dp.cuh's SubTab<false>).
+struct SmemMixed {
+    alignas(16) int subtab[PSUB_INTS];
+    union Warp {
+        WarpSmem w32;
+        PairWarp wp;
+    } w[WARPS];
+    uint8_t ecodes[WARPS][EAGER_W * EAGER_W + 15];
+};
+
+// 72 registers = 7 CTAs per SM; ptxas's own choice for the fused code is 122 (4 CTAs).  At 72 the 32-bit steady loop
+// runs 57.0 instructions per step (55.4 in k_inspect) and the packed loop 88.6 (as in k_inspect_pair), no spills in
+// either loop (SASS, tools/sass_fastpath.py).
+#ifndef MIXED_MAXREG
+#define MIXED_MAXREG 72
+#endif
+template <int R>
+__device__ __forceinline__ void inspect_one32(const DevParams& P, const Batch& b, const SideArrays& sa,
+                                              const ExecPlan& pl, SideIO& io, int side, int budget) {
+    const int lane = threadIdx.x & 31;
+    __syncwarp();
+    // (re)enter 32-bit mode: the union's column-code ring must hold 32-bit table offsets
+    for (int i = lane; i < CP_RING + BLK; i += 32) io.ws->co[i] = 4 * SubTab<false>::CODE;
+    __syncwarp();
+    setup_side<false>(b, side, io);
+    SideOut o;
+    run_side<R, MODE_INSPECT, true, false, false>(P, io, o);
+    __syncwarp();
+    if (lane == 0) {
+        if (o.flags & SF_ESCALATE) {
+            pl.esc[atomicAdd(&pl.counters[21], 1)] = side;
+        } else {
+            uint32_t flags = o.flags;
+            unsigned long long ops = 0;
+            int nops = 0;
+            if (o.bi <= P.eager_max && o.bj <= P.eager_max && !(flags & (SF_RING | SF_OVERFLOW)) &&
+                !(P.options & OPT_NO_EAGER)) {
+                ops = eager_walk(io.ecodes, o.bi, o.bj, nops);
+                flags |= SF_EAGER;
+            }
+            write_side(P, sa, side, o, flags, ops, nops);
+        }
+    }
+    __syncwarp();
+}
+
+template <int R>
+__global__ void __maxnreg__(MIXED_MAXREG) k_inspect_mixed(DevParams P, PairParams Q, Batch b, int4* ring,
+                                                              int rmask, SideArrays sa, ExecPlan pl,
+                                                              const int* order, int ns, int nlong, int n1,
+                                                              int budget, long long* dbg) {
+    __shared__ SmemMixed sm;
+    // order[0, nlong): the predicted-long head of the order; the first n1 of them (n1 = nlong, or 0 when a
+    // concurrent k_inspect takes them) run here in phase 1 (queue counters[35]); order[nlong, ns) are packed
+    for (int idx = threadIdx.x; idx < PSUB_INTS / 2; idx += blockDim.x) {
+        const int tab = idx / (PSUB_TAB / 8), rem = idx % (PSUB_TAB / 8);
+        const int e = rem / SUBTAB_REP, code = e / 16, a0 = (e / 4) % 4, a1 = e % 4;
+        const unsigned v0 = (unsigned)P.sv[5 * code + a0], v1 = (unsigned)P.sv[5 * code + a1];
+        sm.subtab[2 * idx] = (int)(tab ? v0 << 16 : v0);
+        sm.subtab[2 * idx + 1] = (int)(tab ? v1 << 16 : v1);
+    }
+    __syncthreads();
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int slot = blockIdx.x * WARPS + warp;
+    const unsigned subtab = (unsigned)__cvta_generic_to_shared(sm.subtab);
+    SideIO io;
+    io.ring = ring + (size_t)slot * (size_t)(rmask + 1);
+    io.rmask = rmask;
+    io.ws = &sm.w[warp].w32;
+    io.subtab = subtab;
+    io.ecodes = sm.ecodes[warp];
+    io.eager_max = P.eager_max;
+    io.codes = nullptr;
+    io.stab = nullptr;
+    io.budget = budget;
+    io.ps = nullptr;
+    io.wi = warp;
+    io.K = WARPS;
+    io.maxsw = 0;
+    io.wlim = 0;
+    io.xexp = 0;
+    __shared__ int owns[WARPS];  // redo side claimed by the warp (index into pl.redo), -1: none
+    if (lane == 0) owns[warp] = -1;
+    __syncwarp();
+    volatile int* ctr = pl.counters;
+    volatile int* redo = pl.redo;
+    // claim a pushed redo side (lane 0): index or -1
+    auto claim = [&]() -> int {
+        int c = ctr[34];
+        while (c < ctr[30]) {
+            const int o = atomicCAS(&pl.counters[34], c, c + 1);
+            if (o == c) return c;
+            c = o;
+        }
+        return -1;
+    };
+    // One loop, one 32-bit call site (each inlined copy of the 32-bit inspector costs registers and instructions).
+    // phase 1: predicted-long sides (claimed redo sides first, should any appear); phase 2: packed sides -- a warp
+    // that claims a redo side stops taking packed sides, runs it in 32 bits once both halves are idle, then returns
+    // to the packed queue.  No warp needs to wait for late redo sides: a side is pushed in finish() and the pusher's
+    // very next pop() claims any unclaimed push, so every pushed side has a live claimer; a warp leaves when its
+    // pops find the packed queue empty and nothing left to claim.
+    int phase = 1;
+    long long tph[4] = {clock64(), 0, 0, 0};  // diagnostics: clock at start, end of phase 1, end of phase 2
+    int n32 = 0;
+    for (;;) {
+        int side = -1, c = -1;
+        bool exhausted = false;
+        if (phase == 2) {
+            exhausted = run_pairs<R>(P, Q, b, reinterpret_cast<int2*>(io.ring), rmask, sa, pl, &sm.w[warp].wp,
+                                     subtab, order ? order + nlong : nullptr, ns - nlong, &pl.counters[32], dbg,
+                                     &owns[warp]);
+            __syncwarp();
+            c = owns[warp];
+            __syncwarp();
+            if (lane == 0) owns[warp] = -1;
+        }
+        int next = phase;
+        if (lane == 0) {
+            if (phase == 1) {
+                c = claim();
+                if (c < 0) {
+                    const int item = atomicAdd(&pl.counters[35], 1);
+                    if (item < n1) side = order ? order[item] : item;
+                    else next = 2;
+                }
+            }
+            if (c >= 0)
+                while ((side = redo[c]) < 0) __nanosleep(100);  // the push lands right after the count
+        }
+        __syncwarp();  // lane 0 spun in claim / push waits: reconverge before the collectives
+        side = __shfl_sync(FULL, side, 0);
+        next = __shfl_sync(FULL, next, 0);
+        if (next != phase) tph[phase] = clock64();
+        phase = next;
+        if (side >= 0) {
+            inspect_one32<R>(P, b, sa, pl, io, side, phase == 1 ? budget : INT_MAX);
+            ++n32;
+            continue;
+        }
+        if (exhausted) {
+            tph[2] = clock64();
+            break;
+        }
+    }
+    if (dbg && lane == 0) {
+        long long* d = dbg + 4 * (long long)ns + 4 * slot;
+        d[0] = tph[1] - tph[0];
+        d[1] = tph[2] - tph[0];
+        d[2] = clock64() - tph[0];
+        d[3] = n32;
+    }
+}
+
+int mixed_blocks_per_sm() {
+    int n = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_inspect_mixed<4>, WARPS * 32, 0);
+    return n > 0 ? n : 1;
+}
+
+cudaError_t launch_inspect_mixed(int grid, const DevParams& P, const PairParams& Q, const Batch& b, int4* ring,
+                                 int rmask, const SideArrays& sa, const ExecPlan& pl, const int* order, int nsides,
+                                 int nlong, int n1, int budget, long long* dbg, cudaStream_t st) {
+    if (nsides == 0) return cudaSuccess;
+    k_inspect_mixed<4><<<grid, WARPS * 32, 0, st>>>(P, Q, b, ring, rmask, sa, pl, order, nsides, nlong, n1, budget,
+                                                    dbg);
+    return cudaGetLastError();
+}
+
+int pair_blocks_per_sm() {
+    int n = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_inspect_pair<4>, WARPS * 32, 0);
+    return n > 0 ? n : 1;
+}
+
+cudaError_t launch_inspect_pair(int grid, const DevParams& P, const PairParams& Q, const Batch& b, int2* ring,
+                                int rmask, const SideArrays& sa, const ExecPlan& pl, const int* slist, int nsides,
+                                cudaStream_t st) {
+    if (nsides == 0) return cudaSuccess;
+    k_inspect_pair<4><<<grid, WARPS * 32, 0, st>>>(P, Q, b, ring, rmask, sa, pl, slist, nsides);
+    return cudaGetLastError();
+}
+
+__global__ void k_split(const unsigned* keys, int n, unsigned thr, int* count) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    int lo = 0, hi = n;  // keys descending: first index with key < thr
+    while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (keys[mid] >= thr) lo = mid + 1;
+        else hi = mid;
+    }
+    *count = lo;
+}
+
+cudaError_t launch_split(const unsigned* keys_desc, int n, unsigned thr, int* count, cudaStream_t st) {
+    k_split<<<1, 32, 0, st>>>(keys_desc, n, thr, count);
+    return cudaGetLastError();
+}
+
+// Eager corner codes of a packed-inspector side, recomputed by one thread over [0, i*] x [0, j*] with exactly the
+// inspector's cell rule (dp.cuh; the cone rule only looks inside the rectangle, reading R3), then walked as in
+// inspect_body.  Only sides whose peak lies in the 17x17 corner do any work.
+__global__ void k_eager(DevParams P, Batch b, SideArrays sa, int nsides) {
+    const int side = blockIdx.x * blockDim.x + threadIdx.x;
+    if (side >= nsides) return;
+    uint32_t fl = sa.flags[side];
+    if (!(fl & SF_PAIR)) return;
+    fl &= ~SF_PAIR;
+    const int bi = sa.ti[side], bj = sa.qj[side];
+    if (bi <= P.eager_max && bj <= P.eager_max && !(fl & (SF_RING | SF_OVERFLOW)) && !(P.options & OPT_NO_EAGER)) {
+        SideIO io;
+        setup_side<false>(b, side, io);
+        uint8_t ec[EAGER_W * EAGER_W];
+        int Xr[EAGER_W], Dr[EAGER_W], Wr[EAGER_W];  // row r - 1 (row -1: the strip-0 boundary, dead, W = NEG)
+        for (int c = 0; c <= bj; ++c) {
+            Xr[c] = NEG;
+            Dr[c] = NEG;
+            Wr[c] = NEG;
+        }
+        const int E = P.E, OE = P.OE, Y = P.Y;
+        for (int r = 0; r <= bi; ++r) {
+            const int a = (r >= 1 && r <= io.M) ? base_at(io.Apk, io.Aoff + r - 1) : 0;
+            int xl = NEG, il = NEG, wl = -Y - 1;  // left of column 0 (ramp-up cells: dead, W = -(Y+1))
+            int xdg = r == 0 ? -OE : NEG;          // X(r-1, -1); the origin's diagonal gives H(0,0) = 0
+            for (int c = 0; c <= bj; ++c) {
+                const int code = (c >= 1 && c <= io.N) ? base_at(io.Bpk, io.Boff + c - 1) : 4;
+                const int xu = Xr[c], du = Dr[c], wu = Wr[c];
+                const int h = xdg + P.sv[5 * code + a];
+                const int d = imax(du - E, xu);
+                const int iv = imax(il - E, xl);
+                const int sr = imax(imax(h, d), iv);
+                const int thr = imax(wu, wl);
+                const int xn = sr >= thr ? sr - OE : NEG;
+                const int wn = imax(sr - Y, thr);
+                ec[r * EAGER_W + c] = (uint8_t)cell_code(h, d, iv, du, xu, il, xl, E);
+                xdg = xu;
+                Xr[c] = xn;
+                Dr[c] = d;
+                Wr[c] = wn;
+                xl = xn;
+                il = iv;
+                wl = wn;
+            }
+        }
+        int nops = 0;
+        const unsigned long long ops = eager_walk(ec, bi, bj, nops);
+        fl |= SF_EAGER | ((uint32_t)nops << 8);
+        sa.eops[side] = ops;
+        sa.bound[side] = 0;
+        sa.maxsw[side] = 0;
+    }
+    sa.flags[side] = fl;
+}
+
+cudaError_t launch_eager(const DevParams& P, const Batch& b, const SideArrays& sa, int nsides, cudaStream_t st) {
+    if (nsides == 0) return cudaSuccess;
+    k_eager<<<(nsides + 127) / 128, 128, 0, st>>>(P, b, sa, nsides);
+    return cudaGetLastError();
+}
+
 // Block per side (long sides, escalated by k_inspect): the CTA's warps pipeline the side's strips.
 template <int R, bool NM>
 __global__ void __launch_bounds__(WARPS * 32) k_inspect_block(DevParams P, Batch b, int4* ring, int rmask,

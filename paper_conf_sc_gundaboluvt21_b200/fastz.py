@@ -55,7 +55,8 @@ class fastz_stats(ctypes.Structure):
                 ("bin_counts", ctypes.c_int64 * 8), ("exec_words", ctypes.c_int64), ("cigar_bytes", ctypes.c_int64),
                 ("n_launches", ctypes.c_int64), ("n_waves", ctypes.c_int64), ("n_escalated", ctypes.c_int64),
                 ("n_wide_sides", ctypes.c_int64), ("exec_reserved_words", ctypes.c_int64),
-                ("n_selfcheck_fail", ctypes.c_int64)]
+                ("n_selfcheck_fail", ctypes.c_int64), ("n_packed_sides", ctypes.c_int64),
+                ("n_long_sides", ctypes.c_int64), ("n_redo_sides", ctypes.c_int64)]
 
 
 class fastz_seed_params(ctypes.Structure):

@@ -18,7 +18,7 @@ for k, (a, pred, op, args) in enumerate(ins):
     if a < skip_to:
         continue
     c[op] += 1
-    if op == "BRA" and pred.startswith("@!P") and k > 0 and ins[k - 1][2] == "VOTE.ANY":
+    if op == "BRA" and pred.startswith("@!P") and any(x[2] == "VOTE.ANY" for x in ins[max(0, k - 12):k]):
         t = re.search(r"0x([0-9a-f]+)", args)
         skip_to = int(t.group(1), 16)
 tot = sum(c.values())
