@@ -74,6 +74,7 @@ struct fastz_ctx {
     DBuf woff, soff, roff, bin, list, counters, totals, tmpa, tmpb, tmpc, scan_tmp, wl, wlo;
     DBuf codes, stab, runs, nruns, ciglen, cigar, recs, cells, ring, small, wide, ring2, lpt_tmp, order_tmp, order_buf;
     DBuf ring_pair, redo;  // packed inspector (pair.cuh): two rings of int2 per warp slot; abandoned sides
+    DBuf pdbg;             // FASTZ_PAIR_DEBUG diagnostics
     // seeding (fastz_find_hsps)
     DBuf s_kin, s_kout, s_pin, s_pout, s_start, s_cnt, s_off, s_hits, s_hsp, s_keep, s_sel, s_list, s_list2,
         s_k1, s_k2, s_i1, s_i2, s_flag, s_pos, s_out, s_anch, s_tmp;
@@ -386,7 +387,7 @@ void fastz_destroy(fastz_ctx* c) {
                     &c->s_hits, &c->s_hsp, &c->s_keep, &c->s_sel, &c->s_list, &c->s_list2, &c->s_k1, &c->s_k2,
                     &c->s_i1, &c->s_i2, &c->s_flag, &c->s_pos, &c->s_out, &c->s_anch, &c->s_tmp,
                     &c->r_k1, &c->r_k2, &c->r_i1, &c->r_i2, &c->r_box, &c->r_sc, &c->r_red, &c->r_tmp, &c->r_cnt,
-                    &c->ring_pair, &c->redo};
+                    &c->ring_pair, &c->redo, &c->pdbg};
     for (DBuf* b : bufs) dfree(c, *b);
     if (c->ev_ok)
         for (auto& e : c->ev) cudaEventDestroy(e);
@@ -723,8 +724,8 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
         long long* dbg = nullptr;
         const bool pdebug = getenv("FASTZ_PAIR_DEBUG") != nullptr;
         if (pdebug) {
-            AL(wl, (std::max<int64_t>(ns, 1) + (int64_t)c->grid_mixed * WARPS) * 32);
-            dbg = P_<long long>(c->wl);
+            AL(pdbg, (std::max<int64_t>(ns, 1) + (int64_t)c->grid_mixed * WARPS) * 32);
+            dbg = P_<long long>(c->pdbg);
             CK(cudaMemsetAsync(dbg, 0, (size_t)(ns + (int64_t)c->grid_mixed * WARPS) * 32, st));
         }
         if (nlong > 0) {
