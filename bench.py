@@ -437,7 +437,8 @@ def run_fastz(args, ws, rank, local):
     avg = lambda k: sum(s[k] for s in stages) / len(stages)  # noqa: E731
     line = {
         "metric": "GCUPS", "value": value, "unit": "GCUPS", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
+        "ms_per_step": ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "u16x2+int32",
         "data": "synthetic",
         "config": {"workload": desc, "seeds_per_gpu": n, "target_bp": len(w.T), "query_bp": len(w.Q),
                    "l2": "flushed between timed steps (256 MiB write, untimed)",
@@ -454,18 +455,23 @@ def run_fastz(args, ws, rank, local):
         "secondary": secondary,
         "seeding": seeding,
         "dedup": dedup,
-        "roofline": {"bound": "alu", "kernel": "k_inspect", "achieved": achieved / 1e12, "peak": peak_ops / 1e12,
+        "roofline": {"bound": "alu", "kernel": ("inspector stage: k_inspect_mixed (packed u16x2, two sides per warp) + "
+                                                "k_inspect (predicted-long sides, concurrent stream) + k_eager"
+                                                if st0.get("n_packed_sides", 0) else "k_inspect"),
+                     "achieved": achieved / 1e12, "peak": peak_ops / 1e12,
                      "unit": "Tops/s (INT32 lane ops)", "frac": achieved / peak_ops, "traffic": traffic,
                      "traffic_source": traffic_src, "ops_per_cell": OPS_PER_CELL,
                      "frac_with_ydrop": OPS_PER_CELL_YDROP * cells / (insp_ms * 1e-3) / peak_ops,
                      "inspector_ms": insp_ms, "inspector_share_of_step": insp_ms / ms,
                      "algorithmic": f"{OPS_PER_CELL} int ops per explored cell (P:63, P:346: 4 max + 5 add) x "
-                                    f"{cells} explored cells per launch / mean k_inspect time (CUDA events)",
+                                    f"{cells} explored cells per launch / mean inspector-stage time (CUDA events)",
                      "peak_source": f"measured fastz_int_peak (IMNMX/IADD3/VIADDMNMX chains on the ALU + FMA pipes, "
                                     f"128 lane-ops/clk/SM) at {peak_mhz:.0f} MHz; guide-derived 148 SMs x 4 SMSPs x "
                                     f"2 pipes x 16 lanes/clk x 1.965 GHz = 37.2 T/s"},
         "stages_ms": {k: avg(k) for k in ("ms_upload", "ms_inspect", "ms_bin", "ms_execute", "ms_traceback",
                                           "ms_combine")},
+        "inspector_sides": {"packed": st0.get("n_packed_sides", 0), "long_32bit": st0.get("n_long_sides", 0),
+                            "redone_32bit": st0.get("n_redo_sides", 0)},
         "bins_per_side": st0["bin_counts"][:7], "exec_sides": st0["n_exec_sides"], "eager_sides": st0["n_eager_sides"],
         "exec_words": st0["exec_words"], "exec_reserved_words": st0["exec_reserved_words"],
         "wide_sides": st0["n_wide_sides"], "executor_waves": st0["n_waves"],

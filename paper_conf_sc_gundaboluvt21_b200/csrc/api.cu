@@ -319,7 +319,7 @@ bool use_pair(const fastz_ctx* c, const Batch& b, int64_t ns) {
 // predicted length (k_predict's ungapped walk, bases) from which a side goes to the 32-bit inspector first
 unsigned pair_long_threshold() {
     const char* e = getenv("FASTZ_PAIR_LONG");
-    const long v = e ? atol(e) : 96;
+    const long v = e ? atol(e) : 32;  // swept on C2/C3/C5/C6 (profiles/r2/pair_sweep.jsonl): 24-32 best
     return (unsigned)(v < 0 ? 0 : v);
 }
 
