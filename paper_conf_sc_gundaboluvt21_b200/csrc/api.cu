@@ -75,6 +75,7 @@ struct fastz_ctx {
     DBuf codes, stab, runs, nruns, ciglen, cigar, recs, cells, ring, small, wide, ring2, lpt_tmp, order_tmp, order_buf;
     DBuf ring_pair, redo;  // packed inspector (pair.cuh): two rings of int2 per warp slot; abandoned sides
     DBuf pdbg;             // FASTZ_PAIR_DEBUG diagnostics
+    DBuf phist;            // packed inspector: per warp slot and half, strip history (exact executor reservation)
     // seeding (fastz_find_hsps)
     DBuf s_kin, s_kout, s_pin, s_pout, s_start, s_cnt, s_off, s_hits, s_hsp, s_keep, s_sel, s_list, s_list2,
         s_k1, s_k2, s_i1, s_i2, s_flag, s_pos, s_out, s_anch, s_tmp;
@@ -303,6 +304,7 @@ bool pair_params(const DevParams& d, PairParams& q) {
     q.WoutT = -d.Y - 1;
     const char* e = getenv("FASTZ_PAIR_ESCAPE");
     q.esc_strips = e ? std::max(1, atoi(e)) : 16;
+    q.hist = nullptr;
     return true;
 }
 
@@ -387,7 +389,7 @@ void fastz_destroy(fastz_ctx* c) {
                     &c->s_hits, &c->s_hsp, &c->s_keep, &c->s_sel, &c->s_list, &c->s_list2, &c->s_k1, &c->s_k2,
                     &c->s_i1, &c->s_i2, &c->s_flag, &c->s_pos, &c->s_out, &c->s_anch, &c->s_tmp,
                     &c->r_k1, &c->r_k2, &c->r_i1, &c->r_i2, &c->r_box, &c->r_sc, &c->r_red, &c->r_tmp, &c->r_cnt,
-                    &c->ring_pair, &c->redo, &c->pdbg};
+                    &c->ring_pair, &c->redo, &c->pdbg, &c->phist};
     for (DBuf* b : bufs) dfree(c, *b);
     if (c->ev_ok)
         for (auto& e : c->ev) cudaEventDestroy(e);
@@ -741,7 +743,10 @@ int fastz_extend_seeds(fastz_ctx* c, const fastz_seed* seeds, int64_t n, int see
             CK(cudaEventRecord(c->join_ev, c->side_stream));
             pair_launches += 1;
         }
-        CK(launch_inspect_mixed(c->grid_mixed, c->dp, c->pq, b, P_<int4>(c->ring_pair), c->rmask, sa, pl,
+        AL(phist, (size_t)c->grid_mixed * WARPS * 2 * PAIR_HIST * sizeof(int2));
+        PairParams pq = c->pq;
+        pq.hist = P_<int2>(c->phist);
+        CK(launch_inspect_mixed(c->grid_mixed, c->dp, pq, b, P_<int4>(c->ring_pair), c->rmask, sa, pl,
                                 ordered ? order : nullptr, (int)ns, nlong, 0, INT_MAX, dbg, st));
         if (nlong > 0) CK(cudaStreamWaitEvent(st, c->join_ev, 0));
         CK(launch_eager(c->dp, b, sa, (int)ns, st));

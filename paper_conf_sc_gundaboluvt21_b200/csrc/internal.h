@@ -70,8 +70,11 @@ struct PairParams {
     int WoutT;       // W left of column 0 (true value, -(Y+1))
     int esc_strips;  // a packed side still running after this many strips is redone in 32 bits (long sides must
                      // not run packed: a lone packed warp steps ~2x slower than a 32-bit one)
+    int2* hist;      // per warp slot and half: {start column, last step} of strips 0..PAIR_HIST-1 of the current
+                     // side, for the exact executor reservation (nullptr: the 32-bit kernel's bound)
 };
 
+constexpr int PAIR_HIST = 16;
 int pick_R();  // rows per lane (FASTZ_R env: 2, 4 or 8; default 4)
 
 cudaError_t launch_pack(const char* src, int64_t n, uint32_t* fwd, uint32_t* rev, uint16_t* fwdn, uint16_t* revn,

@@ -285,7 +285,13 @@ __device__ __forceinline__ bool run_pairs(const DevParams& P, const PairParams& 
         int2* __restrict__ rg = ringh(h);
         const int start = startv[h], tf = tfin[h] - t0v[h];
         const int e = start + tf - 31;  // lane 31's last column
-        if (lane == 0) hs.steps += tf + 1;
+        int2* const hist = Q.hist ? Q.hist + ((size_t)(blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 2 + h) *
+                                                 PAIR_HIST
+                                  : nullptr;
+        if (lane == 0) {
+            hs.steps += tf + 1;
+            if (hist && hs.s < PAIR_HIST) hist[hs.s] = make_int2(start, tf);
+        }
         bool over = hs.redo != 0;
         int Emax = hs.Emax, Wfar = hs.Wfar;
         uint32_t flags = hs.flags;
@@ -385,6 +391,23 @@ __device__ __forceinline__ bool run_pairs(const DevParams& P, const PairParams& 
             } else {
                 const bool notrim = P.options & OPT_NO_TRIM;
                 const int nstr = hs.s + 1;
+                // Exact executor storage ("allocate ... according to the exact size needed"): the executor's
+                // strip k (k <= i*/H) starts at the same column as the inspector's and runs at most
+                // min(inspector steps, j* - start_k + 31) steps, so its words are bounded by that width exactly.
+                const int speak = bi / H;
+                if (hist && !notrim && speak <= hs.s && speak < PAIR_HIST) {
+                    long long words = 0;
+                    int mx = 0;
+                    for (int k = 0; k <= speak; ++k) {
+                        const int2 hk = hist[k];
+                        const int sp = bj - hk.x > 0 ? bj - hk.x : 0;
+                        const int wk = ((hk.y < sp + 31 ? hk.y : sp + 31) / SPW + 1) * 32;
+                        words += wk;
+                        mx = wk > mx ? wk : mx;
+                    }
+                    bound_words = words;
+                    bound_maxsw = mx;
+                }
                 sa.score[side] = best - (int)Q.Z + P.OE;
                 sa.ti[side] = bi;
                 sa.qj[side] = bj;

@@ -47,7 +47,9 @@ def compare(name, w, **env):
     print(f"{name}: sides {st1['n_sides']} packed {st1['n_packed_sides']} long {st1['n_long_sides']} "
           f"redo {st1['n_redo_sides']} | inspect 32-bit {st0['ms_inspect']:.2f} ms, packed path "
           f"{st1['ms_inspect']:.2f} ms ({st0['ms_inspect'] / max(st1['ms_inspect'], 1e-9):.2f}x) | total "
-          f"{st0['ms_total']:.1f} -> {st1['ms_total']:.1f} ms | {'OK' if not bad else 'MISMATCH ' + str(bad)}",
+          f"{st0['ms_total']:.1f} -> {st1['ms_total']:.1f} ms | reserved/written "
+          f"{st0['exec_reserved_words'] / max(st0['exec_words'], 1):.3f} -> "
+          f"{st1['exec_reserved_words'] / max(st1['exec_words'], 1):.3f} | {'OK' if not bad else 'MISMATCH ' + str(bad)}",
           flush=True)
     return not bad
 
