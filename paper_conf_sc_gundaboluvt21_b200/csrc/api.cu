@@ -292,7 +292,10 @@ bool pair_params(const DevParams& d, PairParams& q) {
     const int64_t Z = negb - negt;
     const int64_t bigt = bigb - Z;
     const int64_t sm = std::max<int64_t>(0, svmax - d.OE);  // largest per-step growth of S
-    const int64_t limt = bigt - d.OE - 4 * sm - 64;        // peak X (true) that abandons the side
+    // peak X (true) that abandons the side: the peak test runs every 2 steps but the half is abandoned at the next
+    // 32-step block boundary, so the margin covers 40 steps of growth -- no value of the half ever reaches BIG_t
+    // (which keeps S - W + 0x8000 and every add inside the half: no carry into the other side's half)
+    const int64_t limt = bigt - d.OE - 40 * sm - 64;
     if (limt < 2000) return false;
     q.Z = (unsigned)Z;
     q.NEGb = (unsigned)negb;
