@@ -382,11 +382,9 @@ __global__ void __launch_bounds__(WARPS * 32) k_inspect_pair(DevParams P, PairPa
     __shared__ SmemPair sm;
     // tables L (low halves) and H (high halves): entry (code, a0, a1), 16 replicas of 8 bytes
     for (int idx = threadIdx.x; idx < PSUB_INTS / 2; idx += blockDim.x) {
-        const int tab = idx / (PSUB_TAB / 8), rem = idx % (PSUB_TAB / 8);
-        const int e = rem / SUBTAB_REP, code = e / 16, a0 = (e / 4) % 4, a1 = e % 4;
-        const unsigned v0 = (unsigned)P.sv[5 * code + a0], v1 = (unsigned)P.sv[5 * code + a1];
-        sm.subtab[2 * idx] = (int)(tab ? v0 << 16 : v0);
-        sm.subtab[2 * idx + 1] = (int)(tab ? v1 << 16 : v1);
+        const int e = idx / SUBTAB_REP, code = e / 16, a0 = (e / 4) % 4, a1 = e % 4;
+        sm.subtab[2 * idx] = P.sv[5 * code + a0];
+        sm.subtab[2 * idx + 1] = P.sv[5 * code + a1];
     }
     for (int idx = threadIdx.x; idx < WARPS * (PCP_RING + BLK); idx += blockDim.x)
         sm.w[idx / (PCP_RING + BLK)].co[idx % (PCP_RING + BLK)] = make_int2(4 * PSUB_CODE, 4 * PSUB_CODE);
@@ -402,7 +400,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_inspect_pair(DevParams P, PairPa
 //   phase 2: the other sides two per warp in the packed inspector (queue counters[32]);
 //   then the sides phase 2 abandoned (value cap, or too many strips: pl.redo, pre-set to -1, counters[30] pushes,
 //   counters[34] claims), in the 32-bit inspector, by whichever warp claims them first (see below).
-// The 32-bit path reads the packed tables' low-half table (the same layout as dp.cuh's SubTab<false>).
+// The 32-bit path reads the packed inspector's table (the same layout as dp.cuh's SubTab<false>).
 struct SmemMixed {
     alignas(16) int subtab[PSUB_INTS];
     union Warp {
@@ -457,11 +455,9 @@ __global__ void __maxnreg__(MIXED_MAXREG) k_inspect_mixed(DevParams P, PairParam
     // order[0, nlong): the predicted-long head of the order; the first n1 of them (n1 = nlong, or 0 when a
     // concurrent k_inspect takes them) run here in phase 1 (queue counters[35]); order[nlong, ns) are packed
     for (int idx = threadIdx.x; idx < PSUB_INTS / 2; idx += blockDim.x) {
-        const int tab = idx / (PSUB_TAB / 8), rem = idx % (PSUB_TAB / 8);
-        const int e = rem / SUBTAB_REP, code = e / 16, a0 = (e / 4) % 4, a1 = e % 4;
-        const unsigned v0 = (unsigned)P.sv[5 * code + a0], v1 = (unsigned)P.sv[5 * code + a1];
-        sm.subtab[2 * idx] = (int)(tab ? v0 << 16 : v0);
-        sm.subtab[2 * idx + 1] = (int)(tab ? v1 << 16 : v1);
+        const int e = idx / SUBTAB_REP, code = e / 16, a0 = (e / 4) % 4, a1 = e % 4;
+        sm.subtab[2 * idx] = P.sv[5 * code + a0];
+        sm.subtab[2 * idx + 1] = P.sv[5 * code + a1];
     }
     __syncthreads();
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;

@@ -26,12 +26,13 @@
 namespace fz {
 
 
-// substitution tables of the packed inspector: entry (code, a0, a1) = {sub(a0, code) + OE, sub(a1, code) + OE} as
-// 16-bit values in the low halves (table L, side A) or high halves (table H, side B), replicated 16x (conflict-free
-// LDS.64, as dp.cuh's SubTab)
+// substitution table of the packed inspector: entry (code, a0, a1) = {sub(a0, code) + OE, sub(a1, code) + OE}
+// (values in [0, 2^16)), replicated 16x (conflict-free LDS.64): dp.cuh's SubTab<false> layout, so the fused
+// kernel's 32-bit path reads the same table; side A's entry lands in the low half and side B's, multiplied by
+// 2^16 in the combining IMAD, in the high half
 constexpr int PSUB_CODE = 16 * SUBTAB_ENTRY;     // bytes per query code (4 x 4 row-pair entries)
 constexpr int PSUB_TAB = 5 * PSUB_CODE;          // bytes per table (codes 0..4)
-constexpr int PSUB_INTS = 2 * PSUB_TAB / 4;
+constexpr int PSUB_INTS = PSUB_TAB / 4;          // one table: side B's values are shifted by the combining IMAD
 
 struct PairHalf {           // strip-level state of one half (shared memory; lane 0 writes, all lanes read)
     const uint32_t* Apk;
@@ -54,6 +55,8 @@ struct PairWarp {
     int4 bout[BLK];           // lane 31's bottom-row outputs, packed
     int bi[2][32], bj[2][32]; // per lane and half: peak position (rare slow path)
     int bfirst[2], blast[2];  // per half: first / last live bottom-row column of the current strip (lane 0 writes)
+    int2 pring[2][32];        // next block's raw ring entries and sequence words, fetched by cp.async during the
+    uint32_t pseq[2][32];     // current block (no registers held; the staging loads no longer stall the warp)
     // per half, current strip: start column, span (N - start), block step at which it began (relative step =
     // tt - t0), termination step (absolute; -1 while running)
     int startv[2], spanv[2], t0v[2], tfin[2];
@@ -104,6 +107,35 @@ __device__ __forceinline__ void pair_boundary(const PairHalf& hs, const int2* __
         w = (unsigned)hs.Wfar;
     }
     if (c > hs.N) w = Q.BIGb;  // columns beyond the query: dead (the 32-bit kernel never computes them)
+}
+
+// boundary + code of half h at column c from the prefetched raw ring entry / sequence word (same rules as
+// pair_boundary / pair_code)
+__device__ __forceinline__ void pair_from_raw(const PairHalf& hs, int2 e, uint32_t word, int c, const PairParams& Q,
+                                              unsigned& x, unsigned& d, unsigned& w, int& code) {
+    if (!hs.active) {
+        x = d = Q.NEGb;
+        w = Q.BIGb;
+        code = 4;
+        return;
+    }
+    if (c <= hs.Emax) {
+        x = (unsigned)e.x & 0xffffu;
+        d = (unsigned)e.x >> 16;
+        w = (unsigned)e.y;
+    } else {
+        x = d = Q.NEGb;
+        w = (unsigned)hs.Wfar;
+    }
+    if (c > hs.N) w = Q.BIGb;
+    code = (c < 1 || c > hs.N) ? 4 : (int)((word >> (((hs.Boff + c - 1) & 15) * 2)) & 3u);
+}
+
+__device__ __forceinline__ void cp_async8(unsigned dst, const void* src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(dst), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async4(unsigned dst, const void* src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(dst), "l"(src) : "memory");
 }
 
 __device__ __forceinline__ int pair_code(const PairHalf& hs, int c) {
@@ -225,7 +257,7 @@ __device__ __forceinline__ bool run_pairs(const DevParams& P, const PairParams& 
             const int r = r0 + k;
             int a = 0;
             if (hs.active && r >= 1 && r <= hs.M) a = base_at(hs.Apk, hs.Aoff + r - 1);
-            const unsigned base = subtab + (unsigned)(h * PSUB_TAB) + (unsigned)((lane & 15) * 8);
+            const unsigned base = subtab + (unsigned)((lane & 15) * 8);
             if (k % 2 == 0) tb[h][k / 2] = base + (unsigned)(a * 4 * SUBTAB_ENTRY);
             else tb[h][k / 2] += (unsigned)(a * SUBTAB_ENTRY);
             const unsigned wv = (hs.active && r <= hs.M) ? (unsigned)hs.Wleft0 : Q.BIGb;
@@ -454,8 +486,8 @@ __device__ __forceinline__ bool run_pairs(const DevParams& P, const PairParams& 
             int l0, l1, h0, h1;
             ld_shared2(fma_add(cA, (int)one, (int)tb[0][p]), l0, l1);
             ld_shared2(fma_add(cB, (int)one, (int)tb[1][p]), h0, h1);
-            w[2 * p] = madu((unsigned)l0, one, (unsigned)h0);
-            w[2 * p + 1] = madu((unsigned)l1, one, (unsigned)h1);
+            w[2 * p] = madu((unsigned)h0, 0x10000u, (unsigned)l0);  // {sub_A, sub_B} halves (no carry: < 2^16)
+            w[2 * p + 1] = madu((unsigned)h1, 0x10000u, (unsigned)l1);
         }
         unsigned xd = xdiag;
         xdiag = xu;
