@@ -210,14 +210,17 @@ __device__ __forceinline__ void setup_side(const Batch& b, int side, SideIO& io)
 
 constexpr int OP_M = 0, OP_I = 1, OP_D = 2;
 
+// the substitution table is sized for the batch's alphabet: the N-free layout (10 KB) leaves 9 KB more of the SM's
+// unified memory to L1 than the N-aware one
+template <bool NM>
 struct SmemDP {
-    alignas(16) int subtab[SUBTAB_INTS];
+    alignas(16) int subtab[SubTab<NM>::INTS];
     WarpSmem w[WARPS];
     uint8_t ecodes[WARPS][EAGER_W * EAGER_W + 15];
 };
 
 template <bool NM>
-__device__ __forceinline__ void smem_init(SmemDP& sm, const DevParams& P) {
+__device__ __forceinline__ void smem_init(SmemDP<NM>& sm, const DevParams& P) {
     using T = SubTab<NM>;
     for (int idx = threadIdx.x; idx < T::INTS / 2; idx += blockDim.x) {
         const int e = idx / SUBTAB_REP, code = e / (T::NB * T::NB), a0 = (e / T::NB) % T::NB, a1 = e % T::NB;
@@ -231,7 +234,8 @@ __device__ __forceinline__ void smem_init(SmemDP& sm, const DevParams& P) {
     __syncthreads();
 }
 
-__device__ __forceinline__ void io_init(SideIO& io, SmemDP& sm, int4* ring, int rmask, int warp_slot, int warp) {
+template <bool NM>
+__device__ __forceinline__ void io_init(SideIO& io, SmemDP<NM>& sm, int4* ring, int rmask, int warp_slot, int warp) {
     io.ring = ring + (size_t)warp_slot * (size_t)(rmask + 1);
     io.rmask = rmask;
     io.ws = &sm.w[warp];
@@ -307,7 +311,7 @@ template <int R, bool NM>
 __device__ __forceinline__ void inspect_body(const DevParams& P, const Batch& b, int4* ring, int rmask,
                                              const SideArrays& sa, const ExecPlan& pl, int budget,
                                              const int* __restrict__ slist, int nlist) {
-    __shared__ SmemDP sm;
+    __shared__ SmemDP<NM> sm;
     smem_init<NM>(sm, P);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     SideIO io;
@@ -662,7 +666,7 @@ cudaError_t launch_eager(const DevParams& P, const Batch& b, const SideArrays& s
 template <int R, bool NM>
 __global__ void __launch_bounds__(WARPS * 32) k_inspect_block(DevParams P, Batch b, int4* ring, int rmask,
                                                                SideArrays sa, ExecPlan pl) {
-    __shared__ SmemDP sm;
+    __shared__ SmemDP<NM> sm;
     __shared__ PipeShared ps;
     __shared__ int cur;
     smem_init<NM>(sm, P);
@@ -690,7 +694,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_inspect_block(DevParams P, Batch
 template <int R, bool NM>
 __global__ void __launch_bounds__(WARPS * 32) k_census(DevParams P, Batch b, int4* ring, int rmask,
                                                         long long* cells, int* counter, const int* slist, int nlist) {
-    __shared__ SmemDP sm;
+    __shared__ SmemDP<NM> sm;
     smem_init<NM>(sm, P);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     SideIO io;
@@ -728,7 +732,7 @@ __global__ void EXECUTE_ATTR k_execute(DevParams P, Batch b, int4* ring, int rma
                                                          SideArrays sa, ExecPlan pl, int lo, int hi, int nblock,
                                                          long long base, Outputs out, int wide) {
     // wide = 1: this launch (the wide ring) runs only the SF_WIDE sides of the range, wide = 0 all others
-    __shared__ SmemDP sm;
+    __shared__ SmemDP<NM> sm;
     __shared__ PipeShared ps;
     __shared__ int cur;
     smem_init<NM>(sm, P);
