@@ -132,3 +132,25 @@ def test_packed_edges(packed):
     assert_ok(bad)
     bad, *_ = compare("A", "A", [(0, 0), (1, 1), (0, 1), (1, 0)])
     assert_ok(bad)
+
+
+@pytest.mark.parametrize("entries", ["64", "256"])
+def test_packed_ring_overflow_goes_wide(packed, entries):
+    """Packed sides whose band outgrows a small boundary ring are flagged (SF_RING) like 32-bit ones and
+    re-inspected with the wide ring by the 32-bit inspector; the batch stays exact."""
+    packed.setenv("FASTZ_RING_ENTRIES", entries)
+    packed.setenv("FASTZ_PAIR_LONG", "100000")  # every side starts packed
+    w = genome.small_pair(91, length=20000, n_seeds=200)
+    bad, g, o, st = compare(w.T, w.Q, w.seeds, census=True)
+    assert_ok(bad)
+    assert st["n_wide_sides"] > 0 and st["n_packed_sides"] == 2 * len(w.seeds)
+
+
+def test_packed_ydrop_1e4_low_identity(packed):
+    """Y just above the default (10^4) on a low-identity pair: wide y-drop blobs, many strips per packed side."""
+    rng = random.Random(10 ** 4)
+    T = rseq(rng, 4000)
+    Q = mutate(rng, T, sub=0.3, indel=0.05)
+    seeds = [(rng.randint(0, 4000), rng.randint(0, len(Q))) for _ in range(60)]
+    bad, *_ = compare(T, Q, seeds, ydrop=10000)
+    assert_ok(bad)
