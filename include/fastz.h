@@ -29,6 +29,11 @@
  * default 80% of free memory), FASTZ_RING_ENTRIES (boundary-ring entries per warp; wider bands take the wide
  * ring), FASTZ_L2_PERSIST=1 (boundary rings in an L2 persisting window during the inspector), FASTZ_SEED_HIT_CAP
  * (seeding scratch), FASTZ_TEST_SELFCHECK=1 (test hook: makes the executor self-check fail).
+ * Packed inspector (two one-sided extensions per warp in 16-bit halves, results identical to the 32-bit
+ * inspector): FASTZ_PAIR (0 never, 1 default: batches with >= 16 sides per warp slot and
+ * parameters the 16-bit arithmetic holds, 2 always), FASTZ_PAIR_LONG (predicted bases from which a side runs in
+ * the 32-bit inspector instead; default 32), FASTZ_PAIR_ESCAPE (strips after which a packed side is redone in
+ * 32 bits; default 16, read at fastz_create), FASTZ_PAIR_DEBUG=1 (per-side and per-warp diagnostics to stderr).
  */
 #ifndef FASTZ_H
 #define FASTZ_H
