@@ -83,7 +83,7 @@ struct fastz_ctx {
     DBuf r_k1, r_k2, r_i1, r_i2, r_box, r_sc, r_red, r_tmp, r_cnt;
     int R = 4, grid = 0, nslots = 0, rmask = 0;
     // packed inspector: launch grid (0 = not built for this context), constants, whether the parameters admit it
-    int grid_pair = 0, grid_mixed = 0;
+    int grid_mixed = 0;
     PairParams pq{};
     bool pair_params_ok = false;
     int64_t n_pair_sides = 0, n_redo_sides = 0, n_long_sides = 0;
@@ -467,7 +467,6 @@ void ctx_finish(fastz_ctx* c) {
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, c->device);
     c->grid = sms * inspector_blocks_per_sm(c->R);
     c->nslots = c->grid * WARPS;
-    c->grid_pair = sms * pair_blocks_per_sm();
     c->grid_mixed = sms * mixed_blocks_per_sm();
     // per-warp boundary ring: the widest explored band is bounded by the query side length; capped (wider
     // bands take the wide ring, fastz_extend_seeds)

@@ -92,9 +92,6 @@ cudaError_t launch_order(const Batch& b, const DevParams& P, int nsides, unsigne
 cudaError_t launch_inspect(int R, int grid, const DevParams& P, const Batch& b, int4* ring, int rmask,
                            const SideArrays& sa, const ExecPlan& pl, int budget, const int* slist, int nlist,
                            cudaStream_t st);
-// packed inspector: sides slist[0, nsides) (all sides when slist is null), two per warp; abandoned sides go to
-// pl.redo (counters[30]).  pair_blocks_per_sm: occupancy of the packed kernel.
-int pair_blocks_per_sm();
 // packed inspection (kernels.cu k_inspect_mixed): order[0, n1) in its 32-bit path (queue counters[35]; n1 = 0 when
 // a concurrent k_inspect takes the predicted-long head order[0, nlong)), order[nlong, nsides) packed two per warp
 // (queue counters[32]), and the sides the packed phase abandons (pl.redo, pre-set to -1; pushes counters[30],
@@ -103,9 +100,6 @@ int mixed_blocks_per_sm();
 cudaError_t launch_inspect_mixed(int grid, const DevParams& P, const PairParams& Q, const Batch& b, int4* ring,
                                  int rmask, const SideArrays& sa, const ExecPlan& pl, const int* order, int nsides,
                                  int nlong, int n1, int budget, long long* dbg, cudaStream_t st);
-cudaError_t launch_inspect_pair(int grid, const DevParams& P, const PairParams& Q, const Batch& b, int2* ring,
-                                int rmask, const SideArrays& sa, const ExecPlan& pl, const int* slist, int nsides,
-                                cudaStream_t st);
 // *count = number of sorted (descending) prediction keys >= thr: the sides the 32-bit inspector takes first
 cudaError_t launch_split(const unsigned* keys_desc, int n, unsigned thr, int* count, cudaStream_t st);
 // eager walk of the packed inspector's sides whose peak lies in the 17x17 corner; clears SF_PAIR

@@ -372,33 +372,6 @@ __global__ void __maxnreg__(INSPECT_N_MAXREG) k_inspect_n(DevParams P, Batch b, 
 }  // namespace fz
 #include "pair.cuh"
 namespace fz {
-// Two sides per warp in 16-bit halves (pair.cuh).  Persistent: each half of each warp pops sides from the queue
-// (slist[0, ns) in order, or all sides when slist is null).
-struct SmemPair {
-    alignas(16) int subtab[PSUB_INTS];
-    PairWarp w[WARPS];
-};
-
-template <int R>
-__global__ void __launch_bounds__(WARPS * 32) k_inspect_pair(DevParams P, PairParams Q, Batch b, int2* ring,
-                                                             int rmask, SideArrays sa, ExecPlan pl, const int* slist,
-                                                             int ns) {
-    __shared__ SmemPair sm;
-    // tables L (low halves) and H (high halves): entry (code, a0, a1), 16 replicas of 8 bytes
-    for (int idx = threadIdx.x; idx < PSUB_INTS / 2; idx += blockDim.x) {
-        const int e = idx / SUBTAB_REP, code = e / 16, a0 = (e / 4) % 4, a1 = e % 4;
-        sm.subtab[2 * idx] = P.sv[5 * code + a0];
-        sm.subtab[2 * idx + 1] = P.sv[5 * code + a1];
-    }
-    for (int idx = threadIdx.x; idx < WARPS * (PCP_RING + BLK); idx += blockDim.x)
-        sm.w[idx / (PCP_RING + BLK)].co[idx % (PCP_RING + BLK)] = make_int2(4 * PSUB_CODE, 4 * PSUB_CODE);
-    __syncthreads();
-    const int warp = threadIdx.x >> 5;
-    int2* rb = ring + (size_t)(blockIdx.x * WARPS + warp) * 2 * (size_t)(rmask + 1);
-    run_pairs<R>(P, Q, b, rb, rmask, sa, pl, &sm.w[warp], (unsigned)__cvta_generic_to_shared(sm.subtab), slist, ns,
-                 &pl.counters[0]);
-}
-
 // One persistent launch for the whole inspection when the packed inspector is on (no tails between phases):
 //   phase 1: the predicted-long sides order[0, nlong) one per warp in the 32-bit inspector (inline eager walk);
 //   phase 2: the other sides two per warp in the packed inspector (queue counters[32]);
@@ -415,7 +388,7 @@ struct SmemMixed {
 };
 
 // 72 registers = 7 CTAs per SM; ptxas's own choice for the fused code is 122 (4 CTAs).  At 72 the 32-bit steady loop
-// runs 57.0 instructions per step (55.4 in k_inspect) and the packed loop 88.6 (as in k_inspect_pair), no spills in
+// runs 57.0 instructions per step (55.4 in k_inspect) and the packed loop 88.6, no spills in
 // either loop (SASS, tools/sass_fastpath.py).
 #ifndef MIXED_MAXREG
 #define MIXED_MAXREG 72
@@ -568,20 +541,6 @@ cudaError_t launch_inspect_mixed(int grid, const DevParams& P, const PairParams&
     if (nsides == 0) return cudaSuccess;
     k_inspect_mixed<4><<<grid, WARPS * 32, 0, st>>>(P, Q, b, ring, rmask, sa, pl, order, nsides, nlong, n1, budget,
                                                     dbg);
-    return cudaGetLastError();
-}
-
-int pair_blocks_per_sm() {
-    int n = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_inspect_pair<4>, WARPS * 32, 0);
-    return n > 0 ? n : 1;
-}
-
-cudaError_t launch_inspect_pair(int grid, const DevParams& P, const PairParams& Q, const Batch& b, int2* ring,
-                                int rmask, const SideArrays& sa, const ExecPlan& pl, const int* slist, int nsides,
-                                cudaStream_t st) {
-    if (nsides == 0) return cudaSuccess;
-    k_inspect_pair<4><<<grid, WARPS * 32, 0, st>>>(P, Q, b, ring, rmask, sa, pl, slist, nsides);
     return cudaGetLastError();
 }
 

@@ -55,8 +55,6 @@ struct PairWarp {
     int4 bout[BLK];           // lane 31's bottom-row outputs, packed
     int bi[2][32], bj[2][32]; // per lane and half: peak position (rare slow path)
     int bfirst[2], blast[2];  // per half: first / last live bottom-row column of the current strip (lane 0 writes)
-    int2 pring[2][32];        // next block's raw ring entries and sequence words, fetched by cp.async during the
-    uint32_t pseq[2][32];     // current block (no registers held; the staging loads no longer stall the warp)
     // per half, current strip: start column, span (N - start), block step at which it began (relative step =
     // tt - t0), termination step (absolute; -1 while running)
     int startv[2], spanv[2], t0v[2], tfin[2];
@@ -107,35 +105,6 @@ __device__ __forceinline__ void pair_boundary(const PairHalf& hs, const int2* __
         w = (unsigned)hs.Wfar;
     }
     if (c > hs.N) w = Q.BIGb;  // columns beyond the query: dead (the 32-bit kernel never computes them)
-}
-
-// boundary + code of half h at column c from the prefetched raw ring entry / sequence word (same rules as
-// pair_boundary / pair_code)
-__device__ __forceinline__ void pair_from_raw(const PairHalf& hs, int2 e, uint32_t word, int c, const PairParams& Q,
-                                              unsigned& x, unsigned& d, unsigned& w, int& code) {
-    if (!hs.active) {
-        x = d = Q.NEGb;
-        w = Q.BIGb;
-        code = 4;
-        return;
-    }
-    if (c <= hs.Emax) {
-        x = (unsigned)e.x & 0xffffu;
-        d = (unsigned)e.x >> 16;
-        w = (unsigned)e.y;
-    } else {
-        x = d = Q.NEGb;
-        w = (unsigned)hs.Wfar;
-    }
-    if (c > hs.N) w = Q.BIGb;
-    code = (c < 1 || c > hs.N) ? 4 : (int)((word >> (((hs.Boff + c - 1) & 15) * 2)) & 3u);
-}
-
-__device__ __forceinline__ void cp_async8(unsigned dst, const void* src) {
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(dst), "l"(src) : "memory");
-}
-__device__ __forceinline__ void cp_async4(unsigned dst, const void* src) {
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(dst), "l"(src) : "memory");
 }
 
 __device__ __forceinline__ int pair_code(const PairHalf& hs, int c) {
