@@ -112,6 +112,46 @@ __device__ __forceinline__ int pair_code(const PairHalf& hs, int c) {
     return base_at(hs.Bpk, hs.Boff + c - 1);
 }
 
+// Peak update of a packed warp (reading R5: strictly better, or equal in a smaller row; columns only grow): the
+// cells of the previous step (p*) and this step (x*) of both halves, in column order.  Returns the new packed
+// per-lane peak and flag bits (bit h: half h moved its peak; bit 2 + h: it reached the value cap).
+__device__ __noinline__ uint2 pair_peak(PairWarp* ws, unsigned p0, unsigned p1, unsigned p2, unsigned p3, unsigned x0,
+                                        unsigned x1, unsigned x2, unsigned x3, unsigned bestP, int tt, unsigned limX) {
+    constexpr int R = 4, H = 32 * R;
+    const int lane = threadIdx.x & 31;
+    const unsigned xs[2][R] = {{p0, p1, p2, p3}, {x0, x1, x2, x3}};
+    unsigned flg = 0;
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+        const int c = ws->startv[h] - ws->t0v[h] + tt - lane;
+        const int r0 = ws->hs[h].s * H + lane * R;
+        unsigned best = half_of(bestP, h);
+        int bi = ws->bi[h][lane], bj = ws->bj[h][lane];
+        bool any = false;
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+#pragma unroll
+            for (int k = 0; k < R; ++k) {
+                const unsigned x = half_of(xs[q][k], h);
+                const int r = r0 + k;
+                const bool better = x > best || (x == best && r < bi);
+                best = better ? x : best;
+                bi = better ? r : bi;
+                bj = better ? c - 1 + q : bj;
+                any |= better;
+            }
+        }
+        if (any) {
+            const unsigned hm = h ? 0xffff0000u : 0x0000ffffu;
+            bestP = (bestP & ~hm) | (best * 0x10001u & hm);
+            ws->bi[h][lane] = bi;
+            ws->bj[h][lane] = bj;
+            flg |= (best >= limX ? 5u : 1u) << h;
+        }
+    }
+    return make_uint2(bestP, flg);
+}
+
 template <int R>
 __device__ __forceinline__ bool run_pairs(const DevParams& P, const PairParams& Q, const Batch& b, int2* ring_base,
                                           int rmask, const SideArrays& sa, const ExecPlan& pl, PairWarp* ws,
@@ -487,34 +527,11 @@ __device__ __forceinline__ bool run_pairs(const DevParams& P, const PairParams& 
 #pragma unroll
             for (int k = 0; k < R; ++k) Xp[k] = X[k];
         } else if (__any_sync(FULL, (sub_add(cacc, bestP, K8) & K8) != 0u)) {
-            // peak (reading R5), rare: scan both steps' cells of both halves in column order
-#pragma unroll 1
-            for (int h = 0; h < 2; ++h) {
-                const int c = startv[h] - t0v[h] + tt - lane;
-                const int r0 = ws->hs[h].s * H + lane * R;
-                unsigned best = half_of(bestP, h);
-                int bi = ws->bi[h][lane], bj = ws->bj[h][lane];
-                bool any = false;
-#pragma unroll
-                for (int q = 0; q < 2; ++q) {
-#pragma unroll
-                    for (int k = 0; k < R; ++k) {
-                        const unsigned x = half_of(q ? X[k] : Xp[k], h);
-                        const int r = r0 + k;
-                        const bool better = x > best || (x == best && r < bi);
-                        best = better ? x : best;
-                        bi = better ? r : bi;
-                        bj = better ? c - 1 + q : bj;
-                        any |= better;
-                    }
-                }
-                if (any) {
-                    bestP = merge(bestP, best * 0x10001u, hmask(h));
-                    ws->bi[h][lane] = bi;
-                    ws->bj[h][lane] = bj;
-                    flg |= (best >= Q.limX ? 5u : 1u) << h;  // moved (bit h), value cap reached (bit 2 + h)
-                }
-            }
+            // peak (reading R5), rare: an out-of-line scan of both steps' cells of both halves, so the fast path's
+            // registers are not pinned around the branch
+            const uint2 r = pair_peak(ws, Xp[0], Xp[1], Xp[2], Xp[3], X[0], X[1], X[2], X[3], bestP, tt, Q.limX);
+            bestP = r.x;
+            flg |= r.y;
         }
         // lane 31 parks its bottom row
         st_shared4_if(is31, sgo + 16u * (unsigned)j, make_int4((int)bq.x, (int)bq.y, (int)bq.z, 0));
