@@ -48,6 +48,9 @@ struct PairHalf {           // strip-level state of one half (shared memory; lan
 };
 
 constexpr int PCP_RING = 64;  // column-code ring of the packed inspector (reads span [t - 31, t + 31])
+#ifndef PAIR_TERM
+#define PAIR_TERM 32  // steps between strip-termination tests of the packed inspector (8, 16 or 32; measured best 32)
+#endif
 
 struct PairWarp {
     int2 co[PCP_RING + BLK];   // column codes of both halves as table byte offsets (+BLK mirrored)
@@ -612,8 +615,14 @@ __device__ __forceinline__ bool run_pairs(const DevParams& P, const PairParams& 
             for (int u = 0; u < STEADY_UNROLL; ++u)
                 step(t + q + u, u & 3, coq + 8u * (unsigned)u, sgo + 16u * (unsigned)(u & ~3),
                      sgi + 16u * (unsigned)(u & ~3), ttbase);
-            term(t + q + STEADY_UNROLL - 1);
-            if (tfin[0] >= 0 && tfin[1] >= 0) break;  // both strips done: finish them at once
+            if ((q & (PAIR_TERM - 8)) == (PAIR_TERM - 8)) {
+                // strip termination every PAIR_TERM steps (relative step PAIR_TERM - 1 mod PAIR_TERM; the SOLO kernel
+                // tests every 8): a later test only computes and parks more cells that are dead either way (past
+                // the termination column every cell of the strip is dead; their parked W is the exact V - Y), so
+                // results are unchanged while the two halves' ballots, shared loads and syncs run 4x less often
+                term(t + q + STEADY_UNROLL - 1);
+                if (tfin[0] >= 0 && tfin[1] >= 0) break;  // both strips done: finish them at once
+            }
         }
     }
     return true;
